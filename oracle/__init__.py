@@ -1,0 +1,158 @@
+"""TEST INFRASTRUCTURE ONLY — the CPU oracle for cuTS subgraph-isomorphism search.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
+/ ``--impl reference`` legs may import this package.  The product package
+(``paper_conf_sc_xiangkshs21_b200``) never imports it and shares no code with it.
+
+Thin ctypes wrapper around ``oracle/cuts_oracle.c`` (plain C, single-threaded;
+see its header for the paper citations and DESIGN.md §2 for the readings).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "cuts_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+ORC_OK, ORC_EINVAL, ORC_ENOMEM, ORC_EUNSUPPORTED = 0, -1, -2, -7
+
+
+class OracleError(RuntimeError):
+    def __init__(self, code: int):
+        super().__init__(f"oracle returned status {code}")
+        self.code = code
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle with gcc (plain -O2; no tuning)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-o", _LIB, _SRC])
+    return _LIB
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        lib = ctypes.CDLL(build())
+        u32p = ctypes.POINTER(ctypes.c_uint32)
+        u64p = ctypes.POINTER(ctypes.c_uint64)
+        lib.oracle_count.argtypes = [ctypes.c_uint32, u64p, u32p, ctypes.c_uint32, u32p, u32p, u32p,
+                                     ctypes.c_uint64, ctypes.c_uint64, u64p, u64p, u64p, u64p]
+        lib.oracle_enumerate.argtypes = [ctypes.c_uint32, u64p, u32p, ctypes.c_uint32, u32p, u32p, u32p,
+                                         ctypes.c_uint64, ctypes.c_uint64, u32p, ctypes.c_uint64, u64p]
+        lib.oracle_order.argtypes = [ctypes.c_uint32, u32p, u32p, u32p]
+        lib.oracle_validate_graph.argtypes = [ctypes.c_uint32, u64p, u32p]
+        lib.oracle_level1_size.argtypes = [ctypes.c_uint32, u64p, ctypes.c_uint32, u64p]
+        lib.oracle_trie_decode.argtypes = [ctypes.c_uint32, u64p, ctypes.POINTER(u32p),
+                                           ctypes.POINTER(u32p), u32p]
+        for f in (lib.oracle_count, lib.oracle_enumerate, lib.oracle_order,
+                  lib.oracle_validate_graph, lib.oracle_level1_size, lib.oracle_trie_decode):
+            f.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+def _p(a, ct):
+    return a.ctypes.data_as(ctypes.POINTER(ct))
+
+
+def _check(rc):
+    if rc != ORC_OK:
+        raise OracleError(rc)
+
+
+def _graph_arrays(g):
+    rp = np.ascontiguousarray(g.row_ptr, dtype=np.uint64)
+    col = np.ascontiguousarray(g.col, dtype=np.uint32)
+    if col.size == 0:
+        col = np.zeros(1, dtype=np.uint32)
+    return rp, col
+
+
+def _query_arrays(q, order):
+    qr, qc = q.csr()
+    if qc.size == 0:
+        qc = np.zeros(1, dtype=np.uint32)
+    o = None if order is None else np.ascontiguousarray(order, dtype=np.uint32)
+    return np.ascontiguousarray(qr), np.ascontiguousarray(qc), o
+
+
+def validate_graph(g) -> bool:
+    rp, col = _graph_arrays(g)
+    return _load().oracle_validate_graph(g.n, _p(rp, ctypes.c_uint64), _p(col, ctypes.c_uint32)) == ORC_OK
+
+
+def order(q) -> list:
+    """The paper's matching order (readings P5/P6)."""
+    qr, qc, _ = _query_arrays(q, None)
+    out = np.zeros(q.k, dtype=np.uint32)
+    _check(_load().oracle_order(q.k, _p(qr, ctypes.c_uint32), _p(qc, ctypes.c_uint32), _p(out, ctypes.c_uint32)))
+    return out.tolist()
+
+
+def count(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 - 1, levels: bool = False):
+    """Exact number of ordered non-induced embeddings (Python int, 128-bit).
+
+    With ``levels=True`` returns ``(count, [|L_0|, |L_1|, ..., |L_k|])`` where
+    |L_j| counts partial paths of j matched vertices (|L_0| is 0).
+    """
+    rp, col = _graph_arrays(g)
+    qr, qc, o = _query_arrays(q, order)
+    lo = np.zeros(1, np.uint64)
+    hi = np.zeros(1, np.uint64)
+    llo = np.zeros(q.k + 1, np.uint64)
+    lhi = np.zeros(q.k + 1, np.uint64)
+    rc = _load().oracle_count(g.n, _p(rp, ctypes.c_uint64), _p(col, ctypes.c_uint32), q.k,
+                              _p(qr, ctypes.c_uint32), _p(qc, ctypes.c_uint32),
+                              None if o is None else _p(o, ctypes.c_uint32),
+                              root_begin, root_end, _p(lo, ctypes.c_uint64), _p(hi, ctypes.c_uint64),
+                              _p(llo, ctypes.c_uint64), _p(lhi, ctypes.c_uint64))
+    _check(rc)
+    total = int(lo[0]) | (int(hi[0]) << 64)
+    if levels:
+        return total, [int(a) | (int(b) << 64) for a, b in zip(llo, lhi)]
+    return total
+
+
+def enumerate_rows(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 - 1,
+                   cap_rows: int | None = None) -> np.ndarray:
+    """All embeddings as a sorted (count, k) uint32 array, row[q] = f(q)."""
+    if cap_rows is None:
+        cap_rows = count(g, q, order, root_begin, root_end)
+    rp, col = _graph_arrays(g)
+    qr, qc, o = _query_arrays(q, order)
+    rows = np.zeros((max(cap_rows, 1), q.k), dtype=np.uint32)
+    nf = np.zeros(1, np.uint64)
+    rc = _load().oracle_enumerate(g.n, _p(rp, ctypes.c_uint64), _p(col, ctypes.c_uint32), q.k,
+                                  _p(qr, ctypes.c_uint32), _p(qc, ctypes.c_uint32),
+                                  None if o is None else _p(o, ctypes.c_uint32),
+                                  root_begin, root_end, _p(rows, ctypes.c_uint32), cap_rows,
+                                  _p(nf, ctypes.c_uint64))
+    _check(rc)
+    return rows[:min(int(nf[0]), cap_rows)]
+
+
+def level1_size(g, min_deg: int) -> int:
+    rp, _ = _graph_arrays(g)
+    out = np.zeros(1, np.uint64)
+    _check(_load().oracle_level1_size(g.n, _p(rp, ctypes.c_uint64), min_deg, _p(out, ctypes.c_uint64)))
+    return int(out[0])
+
+
+def trie_decode(ca_levels, pa_levels) -> np.ndarray:
+    """Decode a (CA, PA) trie (Fig. 3C) into root-to-leaf rows."""
+    L = len(ca_levels)
+    cas = [np.ascontiguousarray(c, dtype=np.uint32) for c in ca_levels]
+    pas = [np.ascontiguousarray(p if p is not None else np.zeros(1), dtype=np.uint32) for p in pa_levels]
+    sizes = np.array([c.size for c in cas], dtype=np.uint64)
+    u32p = ctypes.POINTER(ctypes.c_uint32)
+    ca_arr = (u32p * L)(*[_p(c, ctypes.c_uint32) for c in cas])
+    pa_arr = (u32p * L)(*[_p(p, ctypes.c_uint32) for p in pas])
+    out = np.zeros((int(sizes[-1]), L), dtype=np.uint32)
+    _check(_load().oracle_trie_decode(L, _p(sizes, ctypes.c_uint64), ca_arr, pa_arr, _p(out, ctypes.c_uint32)))
+    return out

@@ -1,0 +1,301 @@
+"""Pins for the CPU oracle (runs with -m "not gpu").
+
+Every test compares the oracle against something other than itself: closed
+forms, brute force over all injective maps, networkx's VF2 monomorphism
+enumerator, scipy sparse traces, or values printed in the paper.
+"""
+import itertools
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from inputs import (er_graph, rmat_graph, complete_graph, cycle_graph, path_graph, star_graph,
+                    grid_graph, petersen_graph, hypercube_graph, complete_bipartite_graph,
+                    graph_from_edges, query_from_edges, named_query, DENSE5, SPARSE5,
+                    dense_family, k_minus)
+from tests import bruteforce
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def falling(x, s):
+    r = 1
+    for i in range(s):
+        r *= (x - i)
+    return r
+
+
+# ----------------------------------------------------------------- closed forms
+@pytest.mark.parametrize("n", [5, 6, 7])
+@pytest.mark.parametrize("qname", ["K3", "C4", "P4", "S3", "K5", "K5-P5", "cricket", "C5", "K1_4"])
+def test_complete_host_any_query(n, qname):
+    """In K_n every injective map is an embedding: n!/(n-k)!."""
+    q = named_query(qname)
+    assert oracle.count(complete_graph(n), q) == math.perm(n, q.k)
+
+
+@pytest.mark.parametrize("n", [3, 4, 5, 8, 11])
+def test_cycles_in_cycle(n):
+    for k in range(3, 9):
+        want = 2 * n if k == n else 0
+        assert oracle.count(cycle_graph(n), named_query(f"C{k}")) == want
+
+
+@pytest.mark.parametrize("n", [4, 6, 9])
+def test_paths_in_cycle(n):
+    for k in range(2, min(n, 8) + 1):
+        assert oracle.count(cycle_graph(n), named_query(f"P{k}")) == 2 * n
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_stars_degree_sequence(seed):
+    """K1,s: sum_v d(v)(d(v)-1)...(d(v)-s+1); P3 = K1,2; K2 = 2m; K1 = n."""
+    g = er_graph(300, 1500, seed)
+    d = g.degrees()
+    for s in (1, 2, 3, 4, 5):
+        assert oracle.count(g, named_query(f"S{s}")) == sum(falling(int(x), s) for x in d)
+    assert oracle.count(g, named_query("P3")) == sum(int(x) * (int(x) - 1) for x in d)
+    assert oracle.count(g, named_query("K1")) == g.n
+    assert oracle.count(g, named_query("P2")) == 2 * g.m
+
+
+def _adj_sparse(g):
+    import scipy.sparse as sp
+    return sp.csr_matrix((np.ones(g.nnz, dtype=np.int64), g.col.astype(np.int64),
+                          g.row_ptr.astype(np.int64)), shape=(g.n, g.n))
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3, 4, 5])
+def test_triangle_and_c4_traces_er1000(seed):
+    """C1 workload (BASELINE configs[0]): K3 = tr(A^3); C4 = tr(A^4) - 2 sum d^2 + sum d."""
+    g = er_graph(1000, 4000, seed)
+    A = _adj_sparse(g)
+    A2 = A @ A
+    tr3 = int((A2.multiply(A)).sum())
+    tr4 = int((A2.multiply(A2)).sum())
+    d = g.degrees()
+    assert oracle.count(g, named_query("K3")) == tr3
+    assert oracle.count(g, named_query("C4")) == tr4 - 2 * int((d * d).sum()) + int(d.sum())
+
+
+def test_traces_rmat12():
+    g = rmat_graph(10, 4, 0.57, 0.19, 0.19, seed=3)
+    A = _adj_sparse(g)
+    A2 = A @ A
+    d = g.degrees()
+    assert oracle.count(g, named_query("K3")) == int((A2.multiply(A)).sum())
+    assert oracle.count(g, named_query("C4")) == int((A2.multiply(A2)).sum()) - 2 * int((d * d).sum()) + int(d.sum())
+
+
+def test_structured_hosts():
+    assert oracle.count(petersen_graph(), named_query("C5")) == 120
+    assert oracle.count(petersen_graph(), named_query("K3")) == 0
+    assert oracle.count(petersen_graph(), named_query("C4")) == 0
+    assert oracle.count(hypercube_graph(3), named_query("C4")) == 48
+    for a, b in [(2, 3), (3, 4), (4, 4)]:
+        assert oracle.count(complete_bipartite_graph(a, b), named_query("C4")) == 2 * a * (a - 1) * b * (b - 1)
+    grid = grid_graph(4, 4)
+    assert oracle.count(grid, named_query("P3")) == 104
+    assert oracle.count(grid, named_query("P4")) == 232
+
+
+def test_fig2_mesh_chain_levels():
+    """Fig. 2: 4x4 mesh, 4-vertex chain.  The paper prints 16 and 48
+    candidates at depths 1 and 2 (exact); its depth-3/4 values 96/192 are
+    schematic (reading P19), so depths 3/4 are pinned by brute force instead."""
+    g = grid_graph(4, 4)
+    q = named_query("P4")
+    S = oracle.order(q)
+    total, lv = oracle.count(g, q, levels=True)
+    assert lv[1] == 16 and lv[2] == 48
+    assert lv == bruteforce.level_sizes(g, q, S)
+    assert total == lv[4] == 232
+
+
+# ------------------------------------------------------------------ brute force
+def _tiny_graphs():
+    gs = [er_graph(8, 14, s) for s in (1, 2, 3)] + [er_graph(9, 20, 4), er_graph(7, 18, 5)]
+    gs.append(graph_from_edges(8, [(0, 1), (1, 2), (2, 0), (2, 3), (3, 4), (4, 5), (5, 3), (6, 7)]))
+    return gs
+
+
+@pytest.mark.parametrize("gi", range(6))
+def test_bruteforce_all_5vertex_queries(gi):
+    g = _tiny_graphs()[gi]
+    for q in DENSE5 + SPARSE5:
+        want = bruteforce.embeddings(g, q)
+        assert oracle.count(g, q) == len(want), q.name
+        rows = oracle.enumerate_rows(g, q)
+        assert [tuple(r) for r in rows.tolist()] == want, q.name
+
+
+@pytest.mark.parametrize("gi", range(6))
+def test_bruteforce_level_sizes(gi):
+    g = _tiny_graphs()[gi]
+    for q in [named_query("K3"), named_query("C4"), named_query("P4"), DENSE5[2], SPARSE5[2], SPARSE5[6]]:
+        S = oracle.order(q)
+        _, lv = oracle.count(g, q, levels=True)
+        assert lv == bruteforce.level_sizes(g, q, S), q.name
+
+
+def test_bruteforce_small_queries_k1_to_4():
+    g = er_graph(9, 16, 7)
+    for q in [named_query("K1"), named_query("P2"), named_query("P3"), named_query("K3"),
+              named_query("S3"), named_query("C4"), named_query("K4"),
+              query_from_edges(4, [(0, 1), (1, 2), (2, 0), (2, 3)])]:
+        assert oracle.count(g, q) == len(bruteforce.embeddings(g, q)), q.name
+
+
+# ---------------------------------------------------------------- networkx VF2
+def _nx(g):
+    import networkx as nx
+    G = nx.Graph()
+    G.add_nodes_from(range(g.n))
+    G.add_edges_from(g.edge_list().tolist())
+    return G
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_networkx_vf2_monomorphisms(seed):
+    """Library routine: networkx GraphMatcher.subgraph_monomorphisms_iter (VF2)."""
+    from networkx.algorithms import isomorphism
+    g = er_graph(30, 100, seed)
+    G = _nx(g)
+    for q in DENSE5[4:] + SPARSE5[:3] + [named_query("C4"), named_query("K4")]:
+        Q = _nx(type(g)(n=q.k, row_ptr=q.csr()[0].astype(np.uint64), col=q.csr()[1]))
+        gm = isomorphism.GraphMatcher(G, Q)
+        # mapping is data->query; convert to rows indexed by query vertex
+        rows = sorted(tuple(inv[qv] for qv in range(q.k))
+                      for m in gm.subgraph_monomorphisms_iter()
+                      for inv in [{v: u for u, v in m.items()}])
+        got = [tuple(r) for r in oracle.enumerate_rows(g, q).tolist()]
+        assert got == rows, q.name
+
+
+# ------------------------------------------------------------------- invariants
+def _aut(q):
+    qe = {(u, v) for u, v in q.edges} | {(v, u) for u, v in q.edges}
+    return sum(all((p[u], p[v]) in qe for u, v in q.edges) for p in itertools.permutations(range(q.k)))
+
+
+def test_automorphism_divides_count():
+    g = rmat_graph(8, 4, 0.57, 0.19, 0.19, seed=2)
+    for q in DENSE5 + SPARSE5:
+        c = oracle.count(g, q)
+        assert c % _aut(q) == 0, q.name
+
+
+def _valid_orders(q):
+    qe = {(u, v) for u, v in q.edges} | {(v, u) for u, v in q.edges}
+    for p in itertools.permutations(range(q.k)):
+        if all(any((p[i], p[j]) in qe for j in range(i)) for i in range(1, q.k)):
+            yield list(p)
+
+
+def test_order_invariance():
+    g = er_graph(60, 300, 3)
+    for q in [DENSE5[5], SPARSE5[0], SPARSE5[4], named_query("C4")]:
+        base = oracle.count(g, q)
+        for o in list(_valid_orders(q))[::7]:
+            assert oracle.count(g, q, order=o) == base, (q.name, o)
+
+
+def test_subquery_monotone():
+    """Q ⊆ Q' on the same vertices => count(Q') <= count(Q) (down the Dense-5 family)."""
+    g = rmat_graph(8, 4, 0.57, 0.19, 0.19, seed=5)
+    fam = sorted(DENSE5, key=lambda q: len(q.edges))
+    cnt = {q.name: oracle.count(g, q) for q in fam}
+    for a in fam:
+        for b in fam:
+            if set(a.edges) <= set(b.edges):
+                assert cnt[b.name] <= cnt[a.name], (a.name, b.name)
+
+
+def test_root_ranges_partition():
+    g = er_graph(200, 1200, 9)
+    q = DENSE5[8]
+    total = oracle.count(g, q)
+    l1 = oracle.level1_size(g, max(q.degrees()))
+    cuts = [0, 17, 50, 51, 120, l1]
+    assert sum(oracle.count(g, q, root_begin=a, root_end=b) for a, b in zip(cuts, cuts[1:])) == total
+
+
+def test_clique_levels_table1_structure():
+    """Table 1 structure: for a K_k query every level j holds
+    j! x (#j-cliques among vertices of degree >= k-1) ordered partial paths."""
+    import networkx as nx
+    g = rmat_graph(9, 4, 0.57, 0.19, 0.19, seed=4)
+    k = 5
+    G = _nx(g)
+    keep = [v for v in range(g.n) if G.degree(v) >= k - 1]
+    H = G.subgraph(keep)
+    cl = [0] * (k + 1)
+    for c in nx.enumerate_all_cliques(H):
+        if len(c) <= k:
+            cl[len(c)] += 1
+    _, lv = oracle.count(g, named_query("K5"), levels=True)
+    for j in range(1, k + 1):
+        assert lv[j] == math.factorial(j) * cl[j]
+
+
+# ---------------------------------------------------------------- order rule
+def test_order_rule_paper():
+    """P:518-530 with min-id ties (readings P5/P6), derived by hand."""
+    assert oracle.order(named_query("cricket")) == [0, 1, 2, 3, 4]          # degs 4,2,2,1,1
+    assert oracle.order(named_query("P5")) == [1, 2, 3, 0, 4]               # degs 1,2,2,2,1
+    assert oracle.order(named_query("K5-K13")) == [4, 1, 2, 3, 0]           # degs 1,3,3,3,4
+    assert oracle.order(named_query("chair")) == [1, 2, 0, 3, 4]            # degs 1,3,2,1,1
+    assert oracle.order(named_query("K5-paw")) == [4, 3, 0, 1, 2]           # degs 2,2,1,3,4
+    assert oracle.order(query_from_edges(4, [(0, 1), (1, 2), (2, 3), (3, 0)])) == [0, 1, 2, 3]
+
+
+def test_root_is_min_candidate_set():
+    """the max-degree root has the smallest level-1 set."""
+    g = rmat_graph(10, 8, seed=2)
+    for q in DENSE5 + SPARSE5:
+        d = q.degrees()
+        root = oracle.order(q)[0]
+        assert all(oracle.level1_size(g, d[root]) <= oracle.level1_size(g, d[v]) for v in range(q.k))
+
+
+# ----------------------------------------------------------------- validation
+def test_validation():
+    assert oracle.validate_graph(er_graph(50, 100, 1))
+    assert oracle.validate_graph(rmat_graph(8, 4, seed=1))
+    from inputs import CSRGraph
+    bad_asym = CSRGraph(n=3, row_ptr=np.array([0, 1, 1, 1], np.uint64), col=np.array([1], np.uint32))
+    bad_loop = CSRGraph(n=2, row_ptr=np.array([0, 1, 1], np.uint64), col=np.array([0], np.uint32))
+    bad_sort = CSRGraph(n=3, row_ptr=np.array([0, 2, 3, 4], np.uint64), col=np.array([2, 1, 0, 0], np.uint32))
+    for g in (bad_asym, bad_loop, bad_sort):
+        assert not oracle.validate_graph(g)
+    with pytest.raises(oracle.OracleError):
+        oracle.count(er_graph(20, 30, 1), query_from_edges(4, [(0, 1), (2, 3)]))   # disconnected Q
+    with pytest.raises(oracle.OracleError):
+        oracle.count(er_graph(20, 30, 1), named_query("P4"), order=[0, 2, 1, 3])   # order not connected
+
+
+# -------------------------------------------------------------- trie (Fig. 3)
+def test_fig3_trie_decode_matches_csf():
+    """Fig. 3: decoding the cuTS (CA, PA) trie gives the same
+    root-to-leaf paths as walking the paper's CSF (nodeid, index) arrays."""
+    fx = json.load(open(os.path.join(GOLDEN, "fig3_trie.json")))
+    got = [tuple(r) for r in oracle.trie_decode(fx["cuts_CA"], fx["cuts_PA"]).tolist()]
+    # independent CSF walk: children of node x at level l are index[l][x]..index[l][x+1]
+    nid, idx = fx["csf_nodeid"], fx["csf_index"]
+    paths = []
+
+    def walk(level, x, prefix):
+        p = prefix + (nid[level][x],)
+        if level == len(nid) - 1:
+            paths.append(p)
+            return
+        for y in range(idx[level][x], idx[level][x + 1]):
+            walk(level + 1, y, p)
+    for x in range(len(nid[0])):
+        walk(0, x, ())
+    assert got == paths
+    assert len(got) == 8 and got[0] == (0, 3, 2, 5) and got[-1] == (1, 2, 3, 4)
