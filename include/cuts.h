@@ -1,0 +1,169 @@
+/*
+ * cuts.h — C ABI of libcuts.so, the B200 (sm_100a) hot path of cuTS
+ * subgraph-isomorphism search (Xiang, Khan, Serra, Halappanavar,
+ * Sukumaran-Rajam, SC '21).  "P:n" cites /root/reference/PAPER.md line n.
+ *
+ * The library counts or enumerates the ORDERED, NON-INDUCED embeddings of a
+ * small connected query graph Q (k <= 8 vertices) in a large undirected data
+ * graph D (Def. 2-4; readings P1/P2 in DESIGN.md):
+ *     Emb(Q, D) = { f : V_Q -> V_D injective | {u,w} in E_Q => {f(u),f(w)} in E_D }.
+ * It does so the paper's way: level-synchronous extension of partial paths
+ * stored in a trie of (parent index, data vertex) levels (Fig. 3C),
+ * each extension being an intersection of backward-neighbour CSR lists
+ * (Alg. 1, Alg. 2 c-intersection P:1019-1031) filtered by
+ * degree (Def. 5) and injectivity, with hybrid BFS/DFS
+ * chunking when a level would not fit.
+ *
+ * Conventions
+ *   - Every call returns cuts_status; no C++ exception crosses the ABI.
+ *     cuts_last_error(ctx) describes the last failing call on ctx.
+ *   - Call order: create -> load_graph -> set_query -> count/enumerate.
+ *     Anything else returns CUTS_ESTATE.
+ *   - Ownership: the CALLER owns every large device buffer (graph, arena,
+ *     enumeration output); the library borrows them and never cudaMallocs.
+ *     Small host arrays (query, order) are copied.
+ *   - Threading: one ctx per host thread.  Work is enqueued on opts.stream and
+ *     every call is host-synchronous (returns when its result is ready).
+ *   - The CUDA path is the only path: there is no CPU fallback.
+ */
+#ifndef CUTS_H
+#define CUTS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CUTS_MAX_K 8
+#define CUTS_ABI_VERSION 1
+
+typedef struct cuts_ctx cuts_ctx;
+
+typedef enum {
+    CUTS_OK = 0,
+    CUTS_EINVAL = -1,       /* bad argument, invalid graph/query/order                  */
+    CUTS_ENOMEM = -2,       /* arena too small (BFS: a level does not fit) */
+    CUTS_ECUDA = -3,        /* a CUDA runtime call failed                               */
+    CUTS_EOVERFLOW = -4,    /* count >= 2^64 (cuts_count); full value in cuts_stats     */
+    CUTS_ETRUNC = -5,       /* enumeration found more rows than cap_rows                */
+    CUTS_ESTATE = -6,       /* call out of order                                        */
+    CUTS_EUNSUPPORTED = -7, /* disconnected query (NEXT-3) or k > 8          */
+    CUTS_ECOMM = -8         /* reserved for the multi-GPU layer                         */
+} cuts_status;
+
+typedef enum {
+    CUTS_BFS = 0,    /* level-synchronous: every level stored whole (Alg. 1);
+                        CUTS_ENOMEM when a level does not fit the arena                    */
+    CUTS_HYBRID = 1  /* BFS inside chunks, DFS over chunks      */
+} cuts_mode;
+
+typedef struct {
+    int       device;       /* CUDA device ordinal                                          */
+    uintptr_t stream;       /* cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream) */
+    void*     arena;        /* caller-owned device scratch: degrees, trie levels, counters  */
+    uint64_t  arena_bytes;  /* hard budget (the paper uses 1/2 of free memory per array,
+                               P:688-691); >= 256-byte aligned base required               */
+    uint64_t  seed;         /* level-1 shuffle; never changes any result        */
+} cuts_opts;
+
+typedef struct {
+    uint32_t k;                        /* query size                                        */
+    uint32_t order[CUTS_MAX_K];        /* matching order S actually used                    */
+    uint64_t level_size[CUTS_MAX_K + 1];  /* |L_j| summed over chunks, j = 0..k; L_k = count
+                                          (low 64 bits); exact and chunk-invariant          */
+    uint64_t count_lo, count_hi;       /* 128-bit embedding count                           */
+    uint64_t level1_canonical;         /* size of the canonical level-1 list (deg filter)   */
+    uint64_t chunks;                   /* extend launches (hybrid chunks x windows)         */
+    uint64_t windows;                  /* plan windows                                      */
+    uint64_t launches;                 /* kernels launched by the last count/enumerate      */
+    uint64_t peak_arena_bytes;         /* high-water mark of the arena stack                */
+    uint64_t items;                    /* candidate items examined (sum of min list sizes)  */
+    double   ms_total;                 /* host wall time of the call                        */
+    double   ms_extend;                /* device time of extend/count kernels (if timing)   */
+    double   ms_plan;                  /* device time of plan + scan kernels (if timing)    */
+    uint64_t extend_launches;          /* launches timed in ms_extend                       */
+    uint64_t alg_bytes_extend;         /* algorithmic bytes of the extend kernels (SURVEY
+                                          §8.d model; only with CUTS_DEBUG_BYTES)           */
+    uint64_t alg_bytes_plan;           /* algorithmic bytes of the plan kernels (ditto)     */
+} cuts_stats;
+
+/* debug / instrumentation flags for cuts_set_debug */
+#define CUTS_DEBUG_TIMING 1u   /* CUDA events around each kernel -> ms_extend / ms_plan     */
+#define CUTS_DEBUG_BYTES  2u   /* per-warp algorithmic byte counters (perturbs timing)      */
+
+/* Create a context bound to opts->device / opts->stream / opts->arena.
+ * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */
+cuts_status cuts_create(cuts_ctx** out, const cuts_opts* opts);
+
+/* Release host resources of ctx (the caller's device buffers are untouched). NULL-safe. */
+void cuts_destroy(cuts_ctx* ctx);
+
+/* Message for the last failing call on ctx (never NULL; "" after success). */
+const char* cuts_last_error(const cuts_ctx* ctx);
+
+/* ABI version (CUTS_ABI_VERSION). */
+int cuts_version(void);
+
+/* Data graph D as symmetric CSR (undirected edges stored both ways,
+ * P:207-209): d_row_ptr u64[n+1], d_col u32[nnz], DEVICE pointers borrowed until
+ * cuts_destroy or the next load.  Rows strictly ascending, no self loops, ids < n.
+ * Derives deg u32[n] into the arena.  validate != 0 runs a device check and
+ * returns CUTS_EINVAL on asymmetry, unsorted rows, duplicates, loops or bad ids. */
+cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz,
+                            const uint64_t* d_row_ptr, const uint32_t* d_col, int validate);
+
+/* Query Q as HOST CSR over 0..k-1 (1 <= k <= 8): row_ptr u32[k+1], col u32[...],
+ * symmetric, no loops/duplicates, connected (else CUTS_EUNSUPPORTED).
+ * order == NULL -> the paper's rule: root = max degree (ties: min id),
+ * then the max-degree vertex adjacent to the matched set (ties: min
+ * id, reading P6).  Else order is a permutation of 0..k-1 in which every
+ * order[i], i >= 1, has a neighbour in order[0..i-1] (else CUTS_EINVAL).
+ * Resets the root range and partition to "all". */
+cuts_status cuts_set_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr,
+                           const uint32_t* col, const uint32_t* order);
+
+/* Restrict the roots to positions [begin, end) of the CANONICAL level-1 list
+ * (vertices with deg >= deg_Q(S[0]) in ascending id, before shuffling; Alg. 1
+ * l.8-11).  end is clamped to the list size.  Default: all. */
+cuts_status cuts_set_root_range(cuts_ctx* ctx, uint64_t begin, uint64_t end);
+
+/* Select a slice of the SHUFFLED level-1 list (after the root range): positions
+ * p in [begin, end) with p % nparts == part.  This is the multi-GPU partition
+ * point (|V_D|/nGPU roots per GPU) and the unit of the dynamic
+ * root-chunk queue.  Default: begin = 0, end = UINT64_MAX, part = 0, nparts = 1. */
+cuts_status cuts_set_root_slice(cuts_ctx* ctx, uint64_t begin, uint64_t end,
+                                uint32_t part, uint32_t nparts);
+
+/* Exact number of ordered non-induced embeddings of Q in D restricted to the
+ * selected roots.  *out = low 64 bits; CUTS_EOVERFLOW if the count is >= 2^64
+ * (full 128-bit value in cuts_stats).  mode: CUTS_BFS or CUTS_HYBRID. */
+cuts_status cuts_count(cuts_ctx* ctx, cuts_mode mode, uint64_t* out);
+
+/* Enumerate embeddings into d_out (DEVICE, cap_rows * k u32): row[q] = f(q) in
+ * QUERY-VERTEX-ID order; row order unspecified (any trie order is valid,
+ * P:700-703).  *n_found is exact; if > cap_rows -> CUTS_ETRUNC and which rows
+ * were written is unspecified. */
+cuts_status cuts_enumerate(cuts_ctx* ctx, cuts_mode mode, uint32_t* d_out,
+                           uint64_t cap_rows, uint64_t* n_found);
+
+/* Stats of the last count/enumerate. */
+cuts_status cuts_get_stats(const cuts_ctx* ctx, cuts_stats* out);
+
+/* Instrumentation flags (CUTS_DEBUG_*); 0 for the timed product path. */
+cuts_status cuts_set_debug(cuts_ctx* ctx, uint32_t flags);
+
+/* Decode a trie (Fig. 3C) held in DEVICE memory: level l (0-based,
+ * l < nlevels <= 8) has sizes[l] entries, candidate ids d_ca[l][x] and parent
+ * indices d_pa[l][x] into level l-1 (d_pa[0] ignored).  Writes, for every entry
+ * x of the last level, the root-to-leaf path as nlevels u32 at d_out[x*nlevels].
+ * sizes / d_ca / d_pa are HOST arrays of length nlevels.  Runs on ctx's stream;
+ * CUTS_EINVAL on a parent index out of range. */
+cuts_status cuts_trie_decode(cuts_ctx* ctx, uint32_t nlevels, const uint64_t* sizes,
+                             const uint32_t* const* d_ca, const uint32_t* const* d_pa,
+                             uint32_t* d_out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUTS_H */

@@ -1,0 +1,196 @@
+"""Thin Python API over the C ABI (argument marshalling only).
+
+PyTorch supplies device memory (the arena, the graph, enumeration output) and
+the stream; every step of the search runs in libcuts.so's CUDA kernels.
+
+    ctx = Cuts(device=0)                 # arena = most of the free HBM
+    ctx.load_graph(row_ptr, col)         # canonical symmetric CSR (numpy or torch)
+    ctx.set_query(q_row_ptr, q_col)      # or ctx.set_query_edges(k, edges)
+    n = ctx.count("hybrid")              # ordered non-induced embeddings
+    rows = ctx.enumerate("bfs", cap)     # (n, k) uint32 on the device, query-id order
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+from . import _lib as L
+
+
+class CutsError(RuntimeError):
+    def __init__(self, status: int, message: str):
+        super().__init__(f"{L.STATUS_NAMES.get(status, status)}: {message}")
+        self.status = status
+        self.message = message
+
+
+_MODES = {"bfs": L.CUTS_BFS, "hybrid": L.CUTS_HYBRID, L.CUTS_BFS: L.CUTS_BFS, L.CUTS_HYBRID: L.CUTS_HYBRID}
+
+
+def _mode(m) -> int:
+    try:
+        return _MODES[m.lower() if isinstance(m, str) else m]
+    except KeyError:
+        raise ValueError(f"mode must be 'bfs' or 'hybrid', got {m!r}") from None
+
+
+def default_arena_bytes(device: int, reserve: int = 4 << 30, fraction: float = 0.9) -> int:
+    free, _ = torch.cuda.mem_get_info(device)
+    return max(1 << 20, int(min(free - reserve, free * fraction)) & ~0xFFFF)
+
+
+class Cuts:
+    """One context on one device: C-ABI handle + torch-owned arena."""
+
+    def __init__(self, device: int = 0, arena_bytes: int | None = None, seed: int = 0x5EED,
+                 stream: torch.cuda.Stream | None = None):
+        self.lib = L.load()
+        if not torch.cuda.is_available():
+            raise RuntimeError("libcuts needs a CUDA device (no CPU fallback)")
+        self.device = torch.device("cuda", device)
+        self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+        if arena_bytes is None:
+            arena_bytes = default_arena_bytes(device)
+        self.arena = torch.empty(int(arena_bytes), dtype=torch.uint8, device=self.device)
+        opts = L.cuts_opts(device=device, stream=self.stream.cuda_stream, arena=self.arena.data_ptr(),
+                           arena_bytes=int(arena_bytes), seed=seed)
+        h = ctypes.c_void_p()
+        rc = self.lib.cuts_create(ctypes.byref(h), ctypes.byref(opts))
+        if rc != 0:
+            raise CutsError(rc, "cuts_create failed")
+        self.h = h
+        self.k = None
+        self._graph = None
+
+    # ----------------------------------------------------------------- utils
+    def _check(self, rc: int, allow=()):
+        if rc != 0 and rc not in allow:
+            raise CutsError(rc, self.lib.cuts_last_error(self.h).decode())
+        return rc
+
+    def close(self):
+        if getattr(self, "h", None):
+            self.lib.cuts_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ------------------------------------------------------------------- API
+    def load_graph(self, row_ptr, col, validate: bool = False):
+        rp = torch.as_tensor(np.asarray(row_ptr, dtype=np.uint64).view(np.int64)) if not torch.is_tensor(row_ptr) else row_ptr
+        cl = torch.as_tensor(np.asarray(col, dtype=np.uint32).view(np.int32)) if not torch.is_tensor(col) else col
+        rp = rp.to(self.device, non_blocking=False).contiguous()
+        cl = cl.to(self.device, non_blocking=False).contiguous()
+        if cl.numel() == 0:
+            cl = torch.zeros(1, dtype=torch.int32, device=self.device)
+            nnz = 0
+        else:
+            nnz = cl.numel()
+        assert rp.element_size() == 8 and cl.element_size() == 4
+        n = rp.numel() - 1
+        self._graph = (rp, cl)   # keep the borrowed buffers alive
+        self._check(self.lib.cuts_load_graph(self.h, n, nnz, rp.data_ptr(), cl.data_ptr(), int(validate)))
+        self.n = n
+        return self
+
+    def load_csr(self, g, validate: bool = False):
+        """Load an ``inputs.CSRGraph``-like object (row_ptr, col attributes)."""
+        return self.load_graph(g.row_ptr, g.col, validate)
+
+    def set_query(self, row_ptr, col, order=None):
+        qr = np.ascontiguousarray(row_ptr, dtype=np.uint32)
+        qc = np.ascontiguousarray(col, dtype=np.uint32)
+        if qc.size == 0:
+            qc = np.zeros(1, dtype=np.uint32)
+        k = qr.size - 1
+        u32p = ctypes.POINTER(ctypes.c_uint32)
+        op = None
+        if order is not None:
+            o = np.ascontiguousarray(order, dtype=np.uint32)
+            op = o.ctypes.data_as(u32p)
+        self._check(self.lib.cuts_set_query(self.h, k, qr.ctypes.data_as(u32p), qc.ctypes.data_as(u32p), op))
+        self.k = k
+        return self
+
+    def set_query_edges(self, k: int, edges, order=None):
+        adj = [[] for _ in range(k)]
+        for u, v in edges:
+            adj[u].append(v)
+            adj[v].append(u)
+        rp = np.zeros(k + 1, dtype=np.uint32)
+        col = []
+        for i in range(k):
+            col += sorted(adj[i])
+            rp[i + 1] = len(col)
+        return self.set_query(rp, np.asarray(col, dtype=np.uint32), order)
+
+    def set_root_range(self, begin: int = 0, end: int = 2**64 - 1):
+        self._check(self.lib.cuts_set_root_range(self.h, begin, end))
+        return self
+
+    def set_root_slice(self, begin: int = 0, end: int = 2**64 - 1, part: int = 0, nparts: int = 1):
+        self._check(self.lib.cuts_set_root_slice(self.h, begin, end, part, nparts))
+        return self
+
+    def set_debug(self, timing: bool = False, bytes_: bool = False):
+        flags = (L.CUTS_DEBUG_TIMING if timing else 0) | (L.CUTS_DEBUG_BYTES if bytes_ else 0)
+        self._check(self.lib.cuts_set_debug(self.h, flags))
+        return self
+
+    def count(self, mode="hybrid") -> int:
+        """Exact count (Python int; values >= 2^64 are returned in full)."""
+        out = ctypes.c_uint64()
+        rc = self._check(self.lib.cuts_count(self.h, _mode(mode), ctypes.byref(out)), allow=(L.CUTS_EOVERFLOW,))
+        if rc == L.CUTS_EOVERFLOW:
+            s = self.stats()
+            return s["count"]
+        return int(out.value)
+
+    def enumerate(self, mode="hybrid", cap_rows: int | None = None, out: torch.Tensor | None = None):
+        """Rows (n_found, k) uint32 (as int32 storage) on the device, query-id order.
+
+        If cap_rows is None a count pass sizes the buffer first."""
+        if cap_rows is None:
+            cap_rows = self.count(mode)
+        if out is None:
+            out = torch.empty((max(int(cap_rows), 1), self.k), dtype=torch.int32, device=self.device)
+        nf = ctypes.c_uint64()
+        rc = self._check(self.lib.cuts_enumerate(self.h, _mode(mode), out.data_ptr(), int(cap_rows), ctypes.byref(nf)),
+                         allow=(L.CUTS_ETRUNC,))
+        self.truncated = rc == L.CUTS_ETRUNC
+        return out[:min(int(nf.value), int(cap_rows))]
+
+    def stats(self) -> dict:
+        s = L.cuts_stats()
+        self._check(self.lib.cuts_get_stats(self.h, ctypes.byref(s)))
+        k = s.k
+        return {
+            "k": k, "order": list(s.order)[:k], "level_size": list(s.level_size)[:k + 1],
+            "count": int(s.count_lo) | (int(s.count_hi) << 64),
+            "level1_canonical": s.level1_canonical, "chunks": s.chunks, "windows": s.windows,
+            "launches": s.launches, "peak_arena_bytes": s.peak_arena_bytes, "items": s.items,
+            "ms_total": s.ms_total, "ms_extend": s.ms_extend, "ms_plan": s.ms_plan,
+            "extend_launches": s.extend_launches, "alg_bytes_extend": s.alg_bytes_extend,
+            "alg_bytes_plan": s.alg_bytes_plan,
+        }
+
+    def trie_decode(self, ca_levels, pa_levels) -> torch.Tensor:
+        """GPU decode of a (CA, PA) trie (Fig. 3C) into root-to-leaf rows."""
+        L_ = len(ca_levels)
+        cas = [torch.as_tensor(np.asarray(c, dtype=np.uint32).view(np.int32)).to(self.device) for c in ca_levels]
+        pas = [torch.as_tensor(np.asarray(p if p is not None else [0], dtype=np.uint32).view(np.int32)).to(self.device)
+               for p in pa_levels]
+        sizes = np.array([c.numel() for c in cas], dtype=np.uint64)
+        out = torch.empty((int(sizes[-1]), L_), dtype=torch.int32, device=self.device)
+        PA = ctypes.c_void_p * L_
+        ca_arr = PA(*[c.data_ptr() for c in cas])
+        pa_arr = PA(*[p.data_ptr() for p in pas])
+        self._check(self.lib.cuts_trie_decode(self.h, L_, sizes.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)),
+                                              ca_arr, pa_arr, out.data_ptr()))
+        return out

@@ -1,0 +1,757 @@
+// cuts.cu — host driver + C ABI of libcuts.so (see include/cuts.h).
+// "P:n" cites /root/reference/PAPER.md line n.  Design: DESIGN.md §4-§5.
+//
+// Memory: everything lives in the caller's arena (P:688-691 uses two halves of
+// cudaMemGetInfo's free space; here the caller decides the budget):
+//   [ctrl block | deg u32[n] | bottom stack ->  ...free...  <- top stack]
+// The bottom stack holds trie levels (persistent while a chunk is being
+// expanded), the top stack holds per-depth window scratch (path, source list,
+// item offsets, scan temp).  HYBRID mode is a DFS over item-range chunks with
+// BFS inside each chunk; BFS mode stores each level whole.
+#include <cuda_runtime.h>
+#include <cub/device/device_scan.cuh>
+#include <cub/device/device_select.cuh>
+#include <thrust/iterator/counting_iterator.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "cuts.h"
+#include "kernels.cuh"
+
+using namespace cuts;
+
+namespace {
+
+constexpr uint64_t kAlign = 256;
+constexpr uint64_t kCtrlBytes = 4096;
+constexpr uint64_t kMaxWindow = 1ull << 22;      // entries per plan window
+constexpr uint64_t kMaxLevel = 0xFFFFFFFFull;    // u32 parent indices
+
+inline uint64_t align_up(uint64_t x) { return (x + kAlign - 1) & ~(kAlign - 1); }
+
+}  // namespace
+
+struct cuts_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    char* arena = nullptr;
+    uint64_t arena_bytes = 0;
+    uint64_t seed = 0;
+    std::string err;
+    int num_sms = 148;
+    unsigned long long* ctrl = nullptr;   // device control words
+    unsigned long long* h_ctrl = nullptr; // pinned host mirror
+    // graph
+    bool has_graph = false;
+    uint32_t n = 0;
+    uint64_t nnz = 0;
+    const uint64_t* row_ptr = nullptr;
+    const uint32_t* col = nullptr;
+    uint32_t* deg = nullptr;
+    uint64_t base_off = 0;                 // first free byte after ctrl + deg
+    // query
+    bool has_query = false;
+    QPlan q{};
+    uint64_t root_begin = 0, root_end = ~0ull;
+    uint64_t slice_begin = 0, slice_end = ~0ull;
+    uint32_t part = 0, nparts = 1;
+    uint32_t debug = 0;
+    // run state
+    uint64_t bot = 0, top = 0, peak = 0;
+    cuts_stats st{};
+    int extend_occ_blocks = 0;
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    std::vector<std::pair<int, int>> ev_ext, ev_plan;
+};
+
+namespace {
+
+cuts_status fail(cuts_ctx* c, cuts_status s, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) c->err = buf;
+    return s;
+}
+
+#define CK(call)                                                                               \
+    do {                                                                                       \
+        cudaError_t e_ = (call);                                                               \
+        if (e_ != cudaSuccess)                                                                 \
+            return fail(ctx, CUTS_ECUDA, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), \
+                        __FILE__, __LINE__);                                                   \
+    } while (0)
+
+#define TRY(expr)                         \
+    do {                                  \
+        cuts_status s_ = (expr);          \
+        if (s_ != CUTS_OK) return s_;     \
+    } while (0)
+
+// ---- arena stacks --------------------------------------------------------
+cuts_status alloc_bot(cuts_ctx* ctx, uint64_t bytes, uint64_t* off) {
+    uint64_t b = align_up(ctx->bot);
+    if (b + bytes > ctx->top) return fail(ctx, CUTS_ENOMEM, "arena exhausted (bottom stack needs %llu B)", (unsigned long long)bytes);
+    *off = b;
+    ctx->bot = b + bytes;
+    ctx->peak = std::max(ctx->peak, ctx->bot + (ctx->arena_bytes - ctx->top));
+    return CUTS_OK;
+}
+cuts_status alloc_top(cuts_ctx* ctx, uint64_t bytes, uint64_t* off) {
+    uint64_t need = align_up(bytes);
+    if (ctx->top < need || ctx->top - need < align_up(ctx->bot))
+        return fail(ctx, CUTS_ENOMEM, "arena exhausted (top stack needs %llu B)", (unsigned long long)bytes);
+    ctx->top -= need;
+    *off = ctx->top;
+    ctx->peak = std::max(ctx->peak, ctx->bot + (ctx->arena_bytes - ctx->top));
+    return CUTS_OK;
+}
+inline uint64_t free_bytes(const cuts_ctx* ctx) {
+    uint64_t b = align_up(ctx->bot);
+    return ctx->top > b ? ctx->top - b : 0;
+}
+
+// ---- events --------------------------------------------------------------
+int next_event(cuts_ctx* ctx) {
+    if (ctx->ev_used == ctx->ev_pool.size()) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return -1;
+        ctx->ev_pool.push_back(e);
+    }
+    return (int)ctx->ev_used++;
+}
+
+// ---- query planning --------------------------------
+bool q_adj(const uint32_t* row, const uint32_t* col, uint32_t a, uint32_t b) {
+    for (uint32_t p = row[a]; p < row[a + 1]; ++p)
+        if (col[p] == b) return true;
+    return false;
+}
+
+cuts_status plan_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row, const uint32_t* col,
+                       const uint32_t* order, QPlan* out) {
+    if (k < 1 || k > CUTS_MAX_K) return fail(ctx, k > CUTS_MAX_K ? CUTS_EUNSUPPORTED : CUTS_EINVAL, "k=%u out of range 1..8", k);
+    if (!row || (row[k] > 0 && !col)) return fail(ctx, CUTS_EINVAL, "null query arrays");
+    if (row[0] != 0) return fail(ctx, CUTS_EINVAL, "query row_ptr[0] != 0");
+    for (uint32_t a = 0; a < k; ++a) {
+        if (row[a + 1] < row[a]) return fail(ctx, CUTS_EINVAL, "query row_ptr not monotone");
+        for (uint32_t p = row[a]; p < row[a + 1]; ++p) {
+            uint32_t b = col[p];
+            if (b >= k || b == a) return fail(ctx, CUTS_EINVAL, "query edge (%u,%u) invalid", a, b);
+            for (uint32_t p2 = row[a]; p2 < p; ++p2)
+                if (col[p2] == b) return fail(ctx, CUTS_EINVAL, "duplicate query edge (%u,%u)", a, b);
+            if (!q_adj(row, col, b, a)) return fail(ctx, CUTS_EINVAL, "query not symmetric at (%u,%u)", a, b);
+        }
+    }
+    uint32_t seen = 1u;   // connectivity (disconnected Q is NEXT-3)
+    for (bool grown = true; grown;) {
+        grown = false;
+        for (uint32_t a = 0; a < k; ++a)
+            if (seen >> a & 1u)
+                for (uint32_t p = row[a]; p < row[a + 1]; ++p)
+                    if (!(seen >> col[p] & 1u)) { seen |= 1u << col[p]; grown = true; }
+    }
+    if (seen != (1u << k) - 1u) return fail(ctx, CUTS_EUNSUPPORTED, "disconnected query graph (P:544-551) is not supported");
+
+    uint32_t S[CUTS_MAX_K];
+    auto qdeg = [&](uint32_t a) { return row[a + 1] - row[a]; };
+    if (order) {
+        uint32_t used = 0;
+        for (uint32_t i = 0; i < k; ++i) {
+            if (order[i] >= k || (used >> order[i] & 1u)) return fail(ctx, CUTS_EINVAL, "order is not a permutation");
+            used |= 1u << order[i];
+            S[i] = order[i];
+        }
+    } else {
+        // root: max degree, ties -> min id; then max degree adjacent
+        // to the matched set, ties -> min id (reading P6)
+        uint32_t used = 0;
+        for (uint32_t i = 0; i < k; ++i) {
+            int pick = -1;
+            for (uint32_t a = 0; a < k; ++a) {
+                if (used >> a & 1u) continue;
+                bool touches = (i == 0);
+                for (uint32_t j = 0; j < i && !touches; ++j) touches = q_adj(row, col, a, S[j]);
+                if (!touches) continue;
+                if (pick < 0 || qdeg(a) > qdeg((uint32_t)pick)) pick = (int)a;
+            }
+            S[i] = (uint32_t)pick;
+            used |= 1u << pick;
+        }
+    }
+    QPlan qp{};
+    qp.k = k;
+    for (uint32_t i = 0; i < k; ++i) {
+        qp.S[i] = S[i];
+        qp.qdeg[i] = qdeg(S[i]);
+        qp.bw[i] = 0;
+        for (uint32_t j = 0; j < i; ++j)
+            if (q_adj(row, col, S[j], S[i])) qp.bw[i] |= 1u << j;
+        if (i > 0 && qp.bw[i] == 0)
+            return fail(ctx, CUTS_EINVAL, "order position %u (query vertex %u) has no backward neighbour", i, S[i]);
+    }
+    *out = qp;
+    return CUTS_OK;
+}
+
+// ---- kernel dispatch -------------------------------------------------------
+struct Window {
+    uint64_t w0;
+    uint32_t W;
+    uint32_t* path;
+    uint64_t* src;
+    uint64_t* ub;
+    uint64_t* offs;
+    void* cub_tmp;
+    size_t cub_bytes;
+    uint64_t total;
+};
+
+template <int J>
+void launch_plan_t(cuts_ctx* ctx, const Graph& g, const Trie& t, const Window& w, int grid) {
+    k_plan<J><<<grid, 256, 0, ctx->stream>>>(g, t, ctx->q, w.w0, w.W, w.path, w.src, w.ub, ctx->ctrl,
+                                             (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0);
+}
+
+void launch_plan(cuts_ctx* ctx, int J, const Graph& g, const Trie& t, const Window& w) {
+    int grid = (int)std::min<uint64_t>((w.W + 1 + 255) / 256, (uint64_t)ctx->num_sms * 8);
+    switch (J) {
+        case 1: launch_plan_t<1>(ctx, g, t, w, grid); break;
+        case 2: launch_plan_t<2>(ctx, g, t, w, grid); break;
+        case 3: launch_plan_t<3>(ctx, g, t, w, grid); break;
+        case 4: launch_plan_t<4>(ctx, g, t, w, grid); break;
+        case 5: launch_plan_t<5>(ctx, g, t, w, grid); break;
+        case 6: launch_plan_t<6>(ctx, g, t, w, grid); break;
+        case 7: launch_plan_t<7>(ctx, g, t, w, grid); break;
+    }
+}
+
+template <int J, int M>
+void launch_extend_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
+                     uint2* out_level, uint32_t* out_rows, uint64_t cap) {
+    uint64_t tiles = (t1 - t0 + kTile - 1) / kTile;
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<J, M>, kTile, 0);
+    if (occ < 1) occ = 1;
+    uint64_t grid = std::min<uint64_t>(tiles, (uint64_t)ctx->num_sms * occ * 4);
+    k_extend<J, M><<<(unsigned)grid, kTile, 0, ctx->stream>>>(g, ctx->q, w.w0, w.W, w.path, w.src, w.offs, t0, t1,
+                                                              out_level, out_rows, cap, ctx->ctrl,
+                                                              (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0);
+}
+
+template <int M>
+void launch_extend_m(cuts_ctx* ctx, int J, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
+                     uint2* out_level, uint32_t* out_rows, uint64_t cap) {
+    switch (J) {
+        case 1: launch_extend_t<1, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 2: launch_extend_t<2, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 3: launch_extend_t<3, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 4: launch_extend_t<4, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 5: launch_extend_t<5, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 6: launch_extend_t<6, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 7: launch_extend_t<7, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+    }
+}
+
+// ---- the level pipeline ----------------------------------------------------
+struct Run {
+    cuts_mode mode;
+    bool enumerate;
+    uint32_t* rows;
+    uint64_t cap_rows;
+    Graph g;
+    Trie t;
+    uint64_t wmax;
+};
+
+uint64_t window_scratch_bytes(uint64_t W, int J, size_t cub_bytes) {
+    return align_up((uint64_t)J * W * 4) + align_up(W * 8) + 2 * align_up((W + 1) * 8) + align_up(cub_bytes) + 4 * kAlign;
+}
+
+cuts_status read_ctrl(cuts_ctx* ctx) {
+    CK(cudaMemcpyAsync(ctx->h_ctrl, ctx->ctrl, kCtrlWords * sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return CUTS_OK;
+}
+
+// plan window [w0, w0+W) of level J: path walk + ub + scan; sets w.total
+cuts_status plan_window(cuts_ctx* ctx, Run& r, int J, Window& w) {
+    int e0 = -1, e1 = -1;
+    if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
+    launch_plan(ctx, J, r.g, r.t, w);
+    CK(cudaGetLastError());
+    CK(cub::DeviceScan::ExclusiveSum(w.cub_tmp, w.cub_bytes, w.ub, w.offs, (int64_t)w.W + 1, ctx->stream));
+    if (ctx->debug & CUTS_DEBUG_TIMING) {
+        e1 = next_event(ctx);
+        CK(cudaEventRecord(ctx->ev_pool[e1], ctx->stream));
+        ctx->ev_plan.push_back({e0, e1});
+    }
+    CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords, w.offs + w.W, sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    w.total = ctx->h_ctrl[kCtrlWords];
+    ctx->st.windows++;
+    ctx->st.launches += 2;
+    ctx->st.items += w.total;
+    return CUTS_OK;
+}
+
+cuts_status extend_range(cuts_ctx* ctx, Run& r, int J, const Window& w, uint64_t t0, uint64_t t1, int mode,
+                         uint2* out, uint64_t cap) {
+    if (t1 <= t0) return CUTS_OK;
+    int e0 = -1;
+    if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
+    if (mode == kWrite) launch_extend_m<kWrite>(ctx, J, r.g, w, t0, t1, out, nullptr, cap);
+    else if (mode == kCount) launch_extend_m<kCount>(ctx, J, r.g, w, t0, t1, nullptr, nullptr, 0);
+    else launch_extend_m<kEnum>(ctx, J, r.g, w, t0, t1, nullptr, r.rows, r.cap_rows);
+    CK(cudaGetLastError());
+    if (ctx->debug & CUTS_DEBUG_TIMING) {
+        int e1 = next_event(ctx);
+        CK(cudaEventRecord(ctx->ev_pool[e1], ctx->stream));
+        ctx->ev_ext.push_back({e0, e1});
+    }
+    ctx->st.chunks++;
+    ctx->st.launches++;
+    return CUTS_OK;
+}
+
+cuts_status alloc_window(cuts_ctx* ctx, int J, uint64_t W, Window* w) {
+    size_t cub_bytes = 0;
+    CK(cub::DeviceScan::ExclusiveSum(nullptr, cub_bytes, (uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)W + 1, ctx->stream));
+    uint64_t off;
+    TRY(alloc_top(ctx, window_scratch_bytes(W, J, cub_bytes), &off));
+    char* p = ctx->arena + off;
+    w->path = (uint32_t*)p; p += align_up((uint64_t)J * W * 4);
+    w->src = (uint64_t*)p; p += align_up(W * 8);
+    w->ub = (uint64_t*)p; p += align_up((W + 1) * 8);
+    w->offs = (uint64_t*)p; p += align_up((W + 1) * 8);
+    w->cub_tmp = p;
+    w->cub_bytes = cub_bytes;
+    return CUTS_OK;
+}
+
+// window size for depth J: bounded so all depths' scratch takes <= 1/8 of the arena
+uint64_t pick_window(cuts_ctx* ctx, uint64_t N) {
+    uint64_t per = (uint64_t)(ctx->q.k) * 4 + 24;   // path + src + ub + offs per entry
+    uint64_t budget = ctx->arena_bytes / 8 / std::max<uint32_t>(1, ctx->q.k - 1);
+    uint64_t w = budget / per;
+    w = std::max<uint64_t>(w, 1);
+    w = std::min<uint64_t>(w, kMaxWindow);
+    return std::min<uint64_t>(w, std::max<uint64_t>(N, 1));
+}
+
+// HYBRID: process entries [0, N) of level J stored at r.t.lv[J] (DFS over chunks)
+cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
+    const int k = (int)ctx->q.k;
+    const bool last = (J == k - 1);
+    const uint64_t top_save = ctx->top;
+    for (uint64_t w0 = 0; w0 < N;) {
+        Window w{};
+        w.w0 = w0;
+        w.W = (uint32_t)std::min<uint64_t>(pick_window(ctx, N), N - w0);
+        TRY(alloc_window(ctx, J, w.W, &w));
+        TRY(plan_window(ctx, r, J, w));
+        if (last) {
+            TRY(extend_range(ctx, r, J, w, 0, w.total, r.enumerate ? kEnum : kCount, nullptr, 0));
+        } else {
+            for (uint64_t t = 0; t < w.total;) {
+                // L_{J+1} chunk takes its share of the free space; deeper stored levels
+                // (J+2 .. k-1) and their window scratch share the rest.
+                uint64_t deeper_scratch = 0;
+                const uint64_t wd = pick_window(ctx, ~0ull);
+                size_t cb = 0;
+                CK(cub::DeviceScan::ExclusiveSum(nullptr, cb, (uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)wd + 1, ctx->stream));
+                for (int d = J + 1; d <= k - 1; ++d) deeper_scratch += window_scratch_bytes(wd, d, cb);
+                uint64_t fb = free_bytes(ctx);
+                uint64_t avail = fb > deeper_scratch ? fb - deeper_scratch : 0;
+                uint64_t share = avail / (uint64_t)(k - 1 - J);
+                uint64_t cap = std::min<uint64_t>(share / sizeof(uint2), kMaxLevel);
+                if (cap == 0) return fail(ctx, CUTS_ENOMEM, "HYBRID: arena too small for level %d (free %llu B)", J + 1, (unsigned long long)fb);
+                uint64_t t1 = std::min<uint64_t>(w.total, t + cap);   // items bound children (ub)
+                uint64_t off;
+                const uint64_t bot_save = ctx->bot;
+                TRY(alloc_bot(ctx, (t1 - t) * sizeof(uint2), &off));
+                uint2* out = (uint2*)(ctx->arena + off);
+                CK(cudaMemsetAsync(ctx->ctrl + kCursor, 0, sizeof(unsigned long long), ctx->stream));
+                TRY(extend_range(ctx, r, J, w, t, t1, kWrite, out, t1 - t));
+                CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
+                CK(cudaStreamSynchronize(ctx->stream));
+                uint64_t size = ctx->h_ctrl[kCursor];
+                if (size > t1 - t) return fail(ctx, CUTS_ENOMEM, "internal: chunk overflow");
+                ctx->st.level_size[J + 1] += size;
+                ctx->bot = off + size * sizeof(uint2);     // shrink to the exact level size
+                if (size) {
+                    r.t.lv[J + 1] = out;
+                    TRY(hybrid_level(ctx, r, J + 1, size));
+                }
+                ctx->bot = bot_save;
+                t = t1;
+            }
+        }
+        ctx->top = top_save;
+        w0 += w.W;
+    }
+    return CUTS_OK;
+}
+
+// BFS: every level stored whole (Alg. 1); ENOMEM when a level does not fit
+cuts_status bfs_levels(cuts_ctx* ctx, Run& r, uint64_t N1) {
+    const int k = (int)ctx->q.k;
+    uint64_t N = N1;
+    for (int J = 1; J <= k - 1 && N > 0; ++J) {
+        const bool last = (J == k - 1);
+        const uint64_t top_save = ctx->top;
+        uint64_t W = pick_window(ctx, N);
+        Window w{};
+        TRY(alloc_window(ctx, J, W, &w));
+        uint2* out = nullptr;
+        uint64_t cap = 0, off = 0;
+        if (!last) {
+            cap = std::min<uint64_t>(free_bytes(ctx) / sizeof(uint2), kMaxLevel);
+            if (cap == 0) return fail(ctx, CUTS_ENOMEM, "BFS: no room for level %d", J + 1);
+            TRY(alloc_bot(ctx, cap * sizeof(uint2), &off));
+            out = (uint2*)(ctx->arena + off);
+            CK(cudaMemsetAsync(ctx->ctrl + kCursor, 0, sizeof(unsigned long long), ctx->stream));
+        }
+        for (uint64_t w0 = 0; w0 < N; w0 += W) {
+            w.w0 = w0;
+            w.W = (uint32_t)std::min<uint64_t>(W, N - w0);
+            TRY(plan_window(ctx, r, J, w));
+            TRY(extend_range(ctx, r, J, w, 0, w.total, last ? (r.enumerate ? kEnum : kCount) : kWrite, out, cap));
+        }
+        if (!last) {
+            CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
+            CK(cudaStreamSynchronize(ctx->stream));
+            uint64_t size = ctx->h_ctrl[kCursor];
+            ctx->st.level_size[J + 1] = size;
+            if (size > cap)
+                return fail(ctx, CUTS_ENOMEM, "BFS: level %d has %llu entries, room for %llu (use CUTS_HYBRID)", J + 1,
+                            (unsigned long long)size, (unsigned long long)cap);
+            ctx->bot = off + size * sizeof(uint2);
+            r.t.lv[J + 1] = out;
+            N = size;
+        }
+        ctx->top = top_save;
+    }
+    return CUTS_OK;
+}
+
+// level 1: canonical list -> root range -> shuffle -> slice
+cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
+    const uint64_t top_save = ctx->top;
+    uint64_t off_canon, off_tmp;
+    TRY(alloc_top(ctx, (uint64_t)ctx->n * 4 + 4, &off_canon));
+    uint32_t* canon = (uint32_t*)(ctx->arena + off_canon);
+    DegAtLeast pred{ctx->deg, ctx->q.qdeg[0]};
+    thrust::counting_iterator<uint32_t> it(0);
+    size_t tmp_bytes = 0;
+    unsigned long long* d_num = ctx->ctrl + kNumSel;
+    CK(cub::DeviceSelect::If(nullptr, tmp_bytes, it, canon, d_num, (int64_t)ctx->n, pred, ctx->stream));
+    TRY(alloc_top(ctx, tmp_bytes, &off_tmp));
+    CK(cub::DeviceSelect::If(ctx->arena + off_tmp, tmp_bytes, it, canon, d_num, (int64_t)ctx->n, pred, ctx->stream));
+    TRY(read_ctrl(ctx));
+    const uint64_t ncanon = ctx->h_ctrl[kNumSel];
+    ctx->st.level1_canonical = ncanon;
+    uint64_t rb = std::min(ctx->root_begin, ncanon), re = std::min(ctx->root_end, ncanon);
+    if (re < rb) re = rb;
+    const uint64_t R = re - rb;
+    // slice of shuffled positions [sb, se) with p % nparts == part
+    uint64_t sb = std::min(ctx->slice_begin, R), se = std::min(ctx->slice_end, R);
+    uint64_t cnt = 0, p0 = 0;
+    if (se > sb) {
+        p0 = sb + ((ctx->part + ctx->nparts - (uint32_t)(sb % ctx->nparts)) % ctx->nparts);
+        cnt = p0 < se ? (se - p0 + ctx->nparts - 1) / ctx->nparts : 0;
+    }
+    uint64_t off_l1;
+    TRY(alloc_bot(ctx, std::max<uint64_t>(cnt, 1) * sizeof(uint2), &off_l1));
+    uint2* L1 = (uint2*)(ctx->arena + off_l1);
+    if (cnt) {
+        Shuffle sh{};
+        sh.R = R;
+        uint32_t bits = 2;
+        while ((1ull << bits) < R) ++bits;
+        if (bits & 1) ++bits;
+        sh.half = bits / 2;
+        sh.mask = (uint32_t)((1ull << sh.half) - 1);
+        uint64_t x = ctx->seed;
+        for (int i = 0; i < 4; ++i) {   // splitmix64 round keys
+            x += 0x9E3779B97F4A7C15ull;
+            uint64_t z = x;
+            z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+            z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+            sh.key[i] = z ^ (z >> 31);
+        }
+        unsigned grid = (unsigned)std::min<uint64_t>((cnt + 255) / 256, (uint64_t)ctx->num_sms * 8);
+        k_level1<<<grid, 256, 0, ctx->stream>>>(canon, rb, sh, p0, ctx->nparts, cnt, L1);
+        CK(cudaGetLastError());
+        ctx->st.launches++;
+    }
+    ctx->st.launches += 2;
+    ctx->top = top_save;
+    r.t.lv[1] = L1;
+    *n1 = cnt;
+    return CUTS_OK;
+}
+
+cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* rows, uint64_t cap_rows) {
+    if (!ctx) return CUTS_EINVAL;
+    if (!ctx->has_graph || !ctx->has_query) return fail(ctx, CUTS_ESTATE, "load_graph and set_query must precede count/enumerate");
+    if (mode != CUTS_BFS && mode != CUTS_HYBRID) return fail(ctx, CUTS_EINVAL, "bad mode %d", (int)mode);
+    if (enumerate && !rows && cap_rows) return fail(ctx, CUTS_EINVAL, "null d_out with cap_rows > 0");
+    auto t_start = std::chrono::steady_clock::now();
+    CK(cudaSetDevice(ctx->device));
+    ctx->st = cuts_stats{};
+    ctx->st.k = ctx->q.k;
+    for (uint32_t i = 0; i < ctx->q.k; ++i) ctx->st.order[i] = ctx->q.S[i];
+    ctx->ev_used = 0;
+    ctx->ev_ext.clear();
+    ctx->ev_plan.clear();
+    ctx->bot = ctx->base_off;
+    ctx->top = ctx->arena_bytes & ~(kAlign - 1);
+    ctx->peak = ctx->bot;
+    CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
+
+    Run r{};
+    r.mode = mode;
+    r.enumerate = enumerate;
+    r.rows = rows;
+    r.cap_rows = cap_rows;
+    r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->n};
+    uint64_t n1 = 0;
+    TRY(build_level1(ctx, r, &n1));
+    ctx->st.level_size[1] = n1;
+    const int k = (int)ctx->q.k;
+    if (k == 1) {
+        if (enumerate && n1 && cap_rows) {
+            unsigned grid = (unsigned)std::min<uint64_t>((n1 + 255) / 256, (uint64_t)ctx->num_sms * 8);
+            k_rows_k1<<<grid, 256, 0, ctx->stream>>>(r.t.lv[1], n1, rows, cap_rows);
+            CK(cudaGetLastError());
+        }
+        ctx->h_ctrl[kCountLo] = n1;
+        ctx->h_ctrl[kCountHi] = 0;
+        ctx->h_ctrl[kEnumCursor] = n1;
+        CK(cudaStreamSynchronize(ctx->stream));
+    } else if (n1 > 0) {
+        if (mode == CUTS_BFS) TRY(bfs_levels(ctx, r, n1));
+        else TRY(hybrid_level(ctx, r, 1, n1));
+        TRY(read_ctrl(ctx));
+    } else {
+        TRY(read_ctrl(ctx));
+    }
+    if (enumerate) {
+        ctx->st.count_lo = ctx->h_ctrl[kEnumCursor];
+        ctx->st.count_hi = 0;
+    } else {
+        ctx->st.count_lo = ctx->h_ctrl[kCountLo];
+        ctx->st.count_hi = ctx->h_ctrl[kCountHi];
+    }
+    if (k > 1) ctx->st.level_size[k] = ctx->st.count_lo;
+    ctx->st.alg_bytes_plan = ctx->h_ctrl[kBytesPlan];
+    ctx->st.alg_bytes_extend = ctx->h_ctrl[kBytesExt];
+    ctx->st.peak_arena_bytes = ctx->peak;
+    if (ctx->debug & CUTS_DEBUG_TIMING) {
+        double ms = 0;
+        for (auto& pr : ctx->ev_ext) {
+            float f = 0;
+            CK(cudaEventElapsedTime(&f, ctx->ev_pool[pr.first], ctx->ev_pool[pr.second]));
+            ms += f;
+        }
+        ctx->st.ms_extend = ms;
+        ctx->st.extend_launches = ctx->ev_ext.size();
+        ms = 0;
+        for (auto& pr : ctx->ev_plan) {
+            float f = 0;
+            CK(cudaEventElapsedTime(&f, ctx->ev_pool[pr.first], ctx->ev_pool[pr.second]));
+            ms += f;
+        }
+        ctx->st.ms_plan = ms;
+    }
+    ctx->st.ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
+    return CUTS_OK;
+}
+
+}  // namespace
+
+// ============================================================== C ABI
+extern "C" {
+
+int cuts_version(void) { return CUTS_ABI_VERSION; }
+
+cuts_status cuts_create(cuts_ctx** out, const cuts_opts* o) {
+    if (!out || !o) return CUTS_EINVAL;
+    *out = nullptr;
+    if (!o->arena || ((uintptr_t)o->arena % kAlign) != 0 || o->arena_bytes < (64u << 10)) return CUTS_EINVAL;
+    cuts_ctx* ctx = new (std::nothrow) cuts_ctx();
+    if (!ctx) return CUTS_ENOMEM;
+    ctx->device = o->device;
+    ctx->stream = (cudaStream_t)o->stream;
+    ctx->arena = (char*)o->arena;
+    ctx->arena_bytes = o->arena_bytes;
+    ctx->seed = o->seed;
+    ctx->ctrl = (unsigned long long*)ctx->arena;
+    ctx->base_off = kCtrlBytes;
+    cudaError_t e = cudaSetDevice(o->device);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, o->device);
+    if (e == cudaSuccess) e = cudaMallocHost((void**)&ctx->h_ctrl, 2 * kCtrlWords * sizeof(unsigned long long));
+    if (e != cudaSuccess) {
+        delete ctx;
+        return CUTS_ECUDA;
+    }
+    *out = ctx;
+    return CUTS_OK;
+}
+
+void cuts_destroy(cuts_ctx* ctx) {
+    if (!ctx) return;
+    for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+    if (ctx->h_ctrl) cudaFreeHost(ctx->h_ctrl);
+    delete ctx;
+}
+
+const char* cuts_last_error(const cuts_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint64_t* d_row_ptr,
+                            const uint32_t* d_col, int validate) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (!d_row_ptr || (nnz && !d_col)) return fail(ctx, CUTS_EINVAL, "null graph pointer");
+    if (n == 0xFFFFFFFFu) return fail(ctx, CUTS_EINVAL, "n must be < 2^32-1");
+    CK(cudaSetDevice(ctx->device));
+    uint64_t deg_bytes = align_up((uint64_t)n * 4 + 4);
+    if (kCtrlBytes + deg_bytes + (16u << 10) > ctx->arena_bytes) return fail(ctx, CUTS_ENOMEM, "arena too small for deg[%u]", n);
+    ctx->has_graph = false;
+    ctx->n = n;
+    ctx->nnz = nnz;
+    ctx->row_ptr = d_row_ptr;
+    ctx->col = d_col;
+    ctx->deg = (uint32_t*)(ctx->arena + kCtrlBytes);
+    ctx->base_off = kCtrlBytes + deg_bytes;
+    if (n) {
+        unsigned grid = (unsigned)std::min<uint64_t>(((uint64_t)n + 255) / 256, (uint64_t)ctx->num_sms * 8);
+        k_degree<<<grid, 256, 0, ctx->stream>>>(d_row_ptr, n, ctx->deg);
+        CK(cudaGetLastError());
+    }
+    // row_ptr[0] == 0 and row_ptr[n] == nnz
+    uint64_t ends[2] = {1, 0};
+    CK(cudaMemcpyAsync(&ends[0], d_row_ptr, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(&ends[1], d_row_ptr + n, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (ends[0] != 0 || ends[1] != nnz) return fail(ctx, CUTS_EINVAL, "row_ptr[0]=%llu row_ptr[n]=%llu nnz=%llu",
+                                                    (unsigned long long)ends[0], (unsigned long long)ends[1], (unsigned long long)nnz);
+    if (validate && n) {
+        CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
+        Graph g{d_row_ptr, d_col, ctx->deg, n};
+        unsigned grid = (unsigned)std::min<uint64_t>(((uint64_t)n * 32 + 255) / 256, (uint64_t)ctx->num_sms * 16);
+        k_validate<<<grid, 256, 0, ctx->stream>>>(g, ctx->ctrl);
+        CK(cudaGetLastError());
+        TRY(read_ctrl(ctx));
+        if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_EINVAL, "graph is not canonical symmetric CSR (sorted, no loops/dups, ids < n)");
+    }
+    ctx->has_graph = true;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr, const uint32_t* col,
+                           const uint32_t* order) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (!ctx->has_graph) return fail(ctx, CUTS_ESTATE, "cuts_load_graph must precede cuts_set_query");
+    QPlan qp{};
+    ctx->has_query = false;
+    TRY(plan_query(ctx, k, row_ptr, col, order, &qp));
+    ctx->q = qp;
+    ctx->root_begin = 0;
+    ctx->root_end = ~0ull;
+    ctx->slice_begin = 0;
+    ctx->slice_end = ~0ull;
+    ctx->part = 0;
+    ctx->nparts = 1;
+    ctx->has_query = true;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_root_range(cuts_ctx* ctx, uint64_t begin, uint64_t end) {
+    if (!ctx) return CUTS_EINVAL;
+    if (!ctx->has_query) return fail(ctx, CUTS_ESTATE, "cuts_set_query must precede cuts_set_root_range");
+    if (end < begin) return fail(ctx, CUTS_EINVAL, "root range end < begin");
+    ctx->root_begin = begin;
+    ctx->root_end = end;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_root_slice(cuts_ctx* ctx, uint64_t begin, uint64_t end, uint32_t part, uint32_t nparts) {
+    if (!ctx) return CUTS_EINVAL;
+    if (!ctx->has_query) return fail(ctx, CUTS_ESTATE, "cuts_set_query must precede cuts_set_root_slice");
+    if (end < begin || nparts == 0 || part >= nparts) return fail(ctx, CUTS_EINVAL, "bad root slice");
+    ctx->slice_begin = begin;
+    ctx->slice_end = end;
+    ctx->part = part;
+    ctx->nparts = nparts;
+    return CUTS_OK;
+}
+
+cuts_status cuts_count(cuts_ctx* ctx, cuts_mode mode, uint64_t* out) {
+    if (!ctx || !out) return CUTS_EINVAL;
+    ctx->err.clear();
+    TRY(run_query(ctx, mode, false, nullptr, 0));
+    *out = ctx->st.count_lo;
+    if (ctx->st.count_hi) return fail(ctx, CUTS_EOVERFLOW, "count >= 2^64 (hi word %llu)", (unsigned long long)ctx->st.count_hi);
+    return CUTS_OK;
+}
+
+cuts_status cuts_enumerate(cuts_ctx* ctx, cuts_mode mode, uint32_t* d_out, uint64_t cap_rows, uint64_t* n_found) {
+    if (!ctx || !n_found) return CUTS_EINVAL;
+    ctx->err.clear();
+    TRY(run_query(ctx, mode, true, d_out, cap_rows));
+    *n_found = ctx->st.count_lo;
+    if (*n_found > cap_rows) return fail(ctx, CUTS_ETRUNC, "found %llu rows, cap %llu", (unsigned long long)*n_found, (unsigned long long)cap_rows);
+    return CUTS_OK;
+}
+
+cuts_status cuts_get_stats(const cuts_ctx* ctx, cuts_stats* out) {
+    if (!ctx || !out) return CUTS_EINVAL;
+    *out = ctx->st;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_debug(cuts_ctx* ctx, uint32_t flags) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->debug = flags;
+    return CUTS_OK;
+}
+
+cuts_status cuts_trie_decode(cuts_ctx* ctx, uint32_t nlevels, const uint64_t* sizes, const uint32_t* const* d_ca,
+                             const uint32_t* const* d_pa, uint32_t* d_out) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (nlevels == 0 || nlevels > CUTS_MAX_K || !sizes || !d_ca || !d_pa) return fail(ctx, CUTS_EINVAL, "bad trie arguments");
+    CK(cudaSetDevice(ctx->device));
+    DecodeArgs a{};
+    a.L = nlevels;
+    for (uint32_t l = 0; l < nlevels; ++l) {
+        a.ca[l] = d_ca[l];
+        a.pa[l] = l ? d_pa[l] : nullptr;
+        a.size[l] = sizes[l];
+        if (!a.ca[l] || (l && sizes[l] && !a.pa[l])) return fail(ctx, CUTS_EINVAL, "null level %u", l);
+    }
+    CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
+    uint64_t n = sizes[nlevels - 1];
+    if (n) {
+        unsigned grid = (unsigned)std::min<uint64_t>((n + 255) / 256, (uint64_t)ctx->num_sms * 8);
+        k_trie_decode<<<grid, 256, 0, ctx->stream>>>(a, d_out, ctx->ctrl);
+        CK(cudaGetLastError());
+    }
+    TRY(read_ctrl(ctx));
+    if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_EINVAL, "parent index out of range");
+    return CUTS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,333 @@
+// kernels.cuh — sm_100a device code for the cuTS hot path.
+// "P:n" cites /root/reference/PAPER.md line n; design in DESIGN.md §4.
+//
+// Pipeline per level j -> j+1 (one window of W entries of the level-j trie):
+//   k_plan<J>      : per entry, walk the trie path (J-1 parent hops),
+//                    pick the smallest backward-neighbour list as the candidate
+//                    source (c-intersection initial set, Alg. 2 l.22-23), emit
+//                    ub(e) = its length (a never-exceeded bound on children).
+//   exclusive scan : offs = prefix(ub)  ->  flat candidate-item space.
+//   k_extend<J,M>  : load-balanced over items (each thread one (entry, candidate)
+//                    pair, so hub lists are split across CTAs): membership of the
+//                    candidate in every other backward list (binary search in the
+//                    sorted CSR row), degree filter (Def. 5),
+//                    injectivity, then warp-aggregated output slots
+//                    (ballot/popc + one atomic per warp) and the write
+//                    of (vertex, parent) into level j+1 — or a count (last level),
+//                    or a full row in query-id order (enumerate).
+#pragma once
+#include <cstdint>
+
+namespace cuts {
+
+constexpr int kMaxK = 8;
+constexpr int kTile = 256;   // items per CTA tile == threads per CTA
+
+struct QPlan {                 // query in matching-order positions
+    uint32_t k;
+    uint32_t S[kMaxK];         // S[i] = query vertex matched at position i
+    uint32_t qdeg[kMaxK];      // deg_Q(S[i])       (degree filter)
+    uint32_t bw[kMaxK];        // bit p set <=> (S[p], S[i]) in E_Q, p < i (next_neigh)
+};
+
+struct Trie {                  // lv[l] = level l (1-based): .x = data vertex, .y = parent index in level l-1
+    const uint2* lv[kMaxK];
+};
+
+struct Graph {
+    const uint64_t* __restrict__ row_ptr;
+    const uint32_t* __restrict__ col;
+    const uint32_t* __restrict__ deg;
+    uint32_t n;
+};
+
+enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
+
+// control block (u64 words in the arena)
+enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
+            kEnumCursor = 6, kNumSel = 7, kCtrlWords = 64 };
+
+__device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
+    if (v == 0) return;
+    unsigned long long old = atomicAdd(lo_hi, v);
+    if (old + v < old) atomicAdd(lo_hi + 1, 1ull);
+}
+
+__device__ __forceinline__ unsigned long long warp_sum(unsigned long long v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// first position in sorted col[b, e) holding value c, or false
+__device__ __forceinline__ bool list_contains(const uint32_t* __restrict__ col, uint64_t b, uint64_t e,
+                                              uint32_t c) {
+    // branch-light lower bound
+    uint64_t len = e - b;
+    const uint32_t* base = col + b;
+    while (len > 1) {
+        uint64_t half = len >> 1;
+        if (__ldg(base + half - 1) < c) base += half;   // move past the lower half
+        len -= half;
+    }
+    return len == 1 && __ldg(base) == c;
+}
+
+// ------------------------------------------------------------------ degrees
+__global__ void k_degree(const uint64_t* __restrict__ row_ptr, uint32_t n, uint32_t* __restrict__ deg) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x)
+        deg[v] = (uint32_t)(row_ptr[v + 1] - row_ptr[v]);
+}
+
+// graph validation: sorted strictly ascending rows, no loops, ids < n, symmetric.
+// one warp per vertex; sets ctrl[kErr] = 1 on any violation.
+__global__ void k_validate(Graph g, unsigned long long* ctrl) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t v = warp; v < g.n; v += nwarps) {
+        uint64_t b = g.row_ptr[v], e = g.row_ptr[v + 1];
+        bool bad = e < b;
+        for (uint64_t p = b + lane; !bad && p < e; p += 32) {
+            uint32_t u = g.col[p];
+            if (u >= g.n || u == v) { bad = true; break; }
+            if (p > b && g.col[p - 1] >= u) { bad = true; break; }
+            if (!list_contains(g.col, g.row_ptr[u], g.row_ptr[u + 1], (uint32_t)v)) { bad = true; break; }
+        }
+        if (__any_sync(0xffffffffu, bad) && lane == 0) atomicExch(ctrl + kErr, 1ull);
+    }
+}
+
+// ---------------------------------------------------------------- level 1
+// canonical level-1 flags: deg(v) >= deg_Q(S[0])  (Alg. 1 l.8-11)
+struct DegAtLeast {
+    const uint32_t* deg; uint32_t t;
+    __host__ __device__ bool operator()(uint32_t v) const { return deg[v] >= t; }
+};
+
+// seeded bijection on [0, R) (4-round Feistel + cycle walking): the randomised
+// partial-path placement of P:916-922 (reading P25: level 1 only, performance only)
+struct Shuffle {
+    uint64_t R; uint32_t half; uint32_t mask; uint64_t key[4];
+    __device__ __forceinline__ static uint32_t mix(uint64_t x) {
+        x ^= x >> 33; x *= 0xff51afd7ed558ccdull; x ^= x >> 33; x *= 0xc4ceb9fe1a85ec53ull; x ^= x >> 33;
+        return (uint32_t)x;
+    }
+    __device__ __forceinline__ uint64_t apply(uint64_t p) const {
+        do {
+            uint32_t l = (uint32_t)(p >> half) & mask, r = (uint32_t)p & mask;
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                uint32_t nl = r;
+                r = l ^ (mix(key[i] ^ r) & mask);
+                l = nl;
+            }
+            p = ((uint64_t)l << half) | r;
+        } while (p >= R);
+        return p;
+    }
+};
+
+// L1[i] = canon[rb + pi(p0 + i*nparts)], i < cnt
+__global__ void k_level1(const uint32_t* __restrict__ canon, uint64_t rb, Shuffle sh, uint64_t p0,
+                         uint32_t nparts, uint64_t cnt, uint2* __restrict__ L1) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        uint64_t p = p0 + i * nparts;
+        L1[i] = make_uint2(canon[rb + sh.apply(p)], 0u);
+    }
+}
+
+// enumerate rows for k == 1
+__global__ void k_rows_k1(const uint2* __restrict__ L1, uint64_t cnt, uint32_t* __restrict__ rows,
+                          uint64_t cap) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt && i < cap;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        rows[i] = L1[i].x;
+}
+
+// ---------------------------------------------------------------- plan
+// J = number of matched positions of the entries (= next position to match).
+template <int J>
+__global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t w0, uint32_t W,
+                                              uint32_t* __restrict__ path_s,
+                                              uint64_t* __restrict__ src_off,
+                                              uint64_t* __restrict__ ub,
+                                              unsigned long long* __restrict__ ctrl, int count_bytes) {
+    const uint32_t bw = q.bw[J];
+    unsigned long long bytes_plan = 0, bytes_ext = 0;
+    for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e <= W; e += gridDim.x * blockDim.x) {
+        if (e == W) { ub[W] = 0; continue; }
+        uint32_t path[J];
+        uint2 cur = t.lv[J][w0 + e];
+        path[J - 1] = cur.x;
+        uint32_t idx = cur.y;
+#pragma unroll
+        for (int p = J - 2; p >= 0; --p) {          // trie walk
+            cur = t.lv[p + 1][idx];
+            path[p] = cur.x;
+            idx = cur.y;
+        }
+        uint64_t best = ~0ull, bsrc = 0, lists = 0;
+#pragma unroll
+        for (int p = 0; p < J; ++p) {
+            if ((bw >> p) & 1u) {
+                uint64_t b = g.row_ptr[path[p]];
+                uint64_t d = g.row_ptr[path[p] + 1] - b;
+                lists += d;
+                if (d < best) { best = d; bsrc = b; }
+            }
+        }
+#pragma unroll
+        for (int p = 0; p < J; ++p) path_s[(size_t)p * W + e] = path[p];
+        src_off[e] = bsrc;
+        ub[e] = best;
+        if (count_bytes) {   // 8 (entry) + 8(J-1) (hops) + 16 per list bound
+            bytes_plan += 8ull + 8ull * (J - 1) + 16ull * __popc(bw);
+            bytes_ext += 4ull * lists;                   // every backward list read once
+        }
+    }
+    if (count_bytes) {
+        bytes_plan = warp_sum(bytes_plan);
+        bytes_ext = warp_sum(bytes_ext);
+        if ((threadIdx.x & 31) == 0) {
+            atomicAdd(ctrl + kBytesPlan, bytes_plan);
+            atomicAdd(ctrl + kBytesExt, bytes_ext);
+        }
+    }
+}
+
+// ---------------------------------------------------------------- extend
+// Items [t0, t1) of the window's flat candidate space (offs = exclusive scan of
+// ub, W+1 entries).  J = matched positions of the parents; the child takes
+// position J.  M selects the output: kWrite -> level J+1 entries (vertex,
+// parent = w0 + e) at ctrl[kCursor] (dropped past cap; the caller sizes cap so
+// that never happens in HYBRID); kCount -> 128-bit count; kEnum -> rows of k u32
+// in query-id order at ctrl[kEnumCursor].
+template <int J, int M>
+__global__ void __launch_bounds__(kTile) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
+                                                  const uint32_t* __restrict__ path_s,
+                                                  const uint64_t* __restrict__ src_off,
+                                                  const uint64_t* __restrict__ offs,
+                                                  uint64_t t0, uint64_t t1,
+                                                  uint2* __restrict__ out_level,
+                                                  uint32_t* __restrict__ out_rows, uint64_t cap,
+                                                  unsigned long long* __restrict__ ctrl, int count_bytes) {
+    __shared__ uint64_t s_offs[kTile + 1];
+    __shared__ uint32_t s_ef;
+    const uint32_t bw = q.bw[J];
+    const uint32_t qd = q.qdeg[J];
+    const int lane = threadIdx.x & 31;
+    unsigned long long my_count = 0, bytes = 0;
+
+    for (uint64_t base = t0 + (uint64_t)blockIdx.x * kTile; base < t1; base += (uint64_t)gridDim.x * kTile) {
+        if (threadIdx.x == 0) {          // last entry e with offs[e] <= base
+            uint32_t lo = 0, hi = W - 1;
+            while (lo < hi) {
+                uint32_t mid = (lo + hi + 1) >> 1;
+                if (offs[mid] <= base) lo = mid; else hi = mid - 1;
+            }
+            s_ef = lo;
+        }
+        __syncthreads();
+        const uint32_t ef = s_ef;
+        for (int x = threadIdx.x; x <= kTile; x += blockDim.x) {
+            uint64_t e = (uint64_t)ef + x;
+            s_offs[x] = e <= W ? offs[e] : ~0ull;
+        }
+        __syncthreads();
+
+        const uint64_t t = base + threadIdx.x;
+        bool ok = false;
+        uint32_t c = 0, e = 0;
+        uint32_t path[J];
+        if (t < t1) {
+            uint64_t start;
+            if (s_offs[kTile] > t) {     // entries have ub >= 1, so the tile's entries fit in smem
+                int lo = 0, hi = kTile - 1;
+                while (lo < hi) {
+                    int mid = (lo + hi + 1) >> 1;
+                    if (s_offs[mid] <= t) lo = mid; else hi = mid - 1;
+                }
+                e = ef + lo;
+                start = s_offs[lo];
+            } else {                      // defensive: global search
+                uint32_t lo = ef, hi = W - 1;
+                while (lo < hi) {
+                    uint32_t mid = (lo + hi + 1) >> 1;
+                    if (offs[mid] <= t) lo = mid; else hi = mid - 1;
+                }
+                e = lo;
+                start = offs[lo];
+            }
+            const uint64_t so = src_off[e];
+            c = g.col[so + (t - start)];
+#pragma unroll
+            for (int p = 0; p < J; ++p) path[p] = path_s[(size_t)p * W + e];
+            bool inj = true;
+#pragma unroll
+            for (int p = 0; p < J; ++p) inj = inj && (path[p] != c);         // injectivity
+            bool inter = inj || count_bytes;
+#pragma unroll
+            for (int p = 0; p < J; ++p) {                                     // c-intersection (Alg. 2)
+                if (((bw >> p) & 1u) && inter) {
+                    uint64_t b = g.row_ptr[path[p]];
+                    if (b != so) inter = list_contains(g.col, b, g.row_ptr[path[p] + 1], c);
+                }
+            }
+            ok = inj && inter && (g.deg[c] >= qd);                            // degree filter (Def. 5)
+            if (count_bytes) bytes += (inter ? 4ull : 0ull) + (ok && M != kCount ? (M == kEnum ? 4ull * q.k : 8ull) : 0ull);
+        }
+        if (M == kCount) {
+            my_count += ok ? 1 : 0;
+        } else {
+            const unsigned m = __ballot_sync(0xffffffffu, ok);
+            const int nsel = __popc(m);
+            unsigned long long pos0 = 0;
+            if (lane == 0 && nsel) pos0 = atomicAdd(ctrl + (M == kWrite ? kCursor : kEnumCursor), (unsigned long long)nsel);
+            pos0 = __shfl_sync(0xffffffffu, pos0, 0);
+            const unsigned long long pos = pos0 + __popc(m & ((1u << lane) - 1u));
+            if (ok && pos < cap) {
+                if (M == kWrite) {
+                    out_level[pos] = make_uint2(c, (uint32_t)(w0 + e));
+                } else {
+                    uint32_t* row = out_rows + pos * q.k;
+#pragma unroll
+                    for (int p = 0; p < J; ++p) row[q.S[p]] = path[p];
+                    row[q.S[J]] = c;
+                }
+            }
+        }
+        __syncthreads();
+    }
+    if (M == kCount) {
+        my_count = warp_sum(my_count);
+        if (lane == 0) add_u128(ctrl + kCountLo, my_count);
+    }
+    if (count_bytes) {
+        bytes = warp_sum(bytes);
+        if (lane == 0) atomicAdd(ctrl + kBytesExt, bytes);
+    }
+}
+
+// ---------------------------------------------------------------- trie decode
+struct DecodeArgs {
+    const uint32_t* ca[kMaxK];
+    const uint32_t* pa[kMaxK];
+    uint64_t size[kMaxK];
+    uint32_t L;
+};
+
+__global__ void k_trie_decode(DecodeArgs a, uint32_t* __restrict__ out, unsigned long long* ctrl) {
+    const uint64_t n = a.size[a.L - 1];
+    for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x < n; x += (uint64_t)gridDim.x * blockDim.x) {
+        uint64_t at = x;
+        for (int l = (int)a.L - 1; l >= 0; --l) {
+            if (at >= a.size[l]) { atomicExch(ctrl + kErr, 1ull); break; }
+            out[x * a.L + l] = a.ca[l][at];
+            if (l > 0) at = a.pa[l][at];
+        }
+    }
+}
+
+}  // namespace cuts

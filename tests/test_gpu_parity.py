@@ -1,0 +1,283 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Integer work, so the bar is bit-exact: counts, per-level trie sizes (same
+matching order on both sides) and sorted embedding rows.  Row order inside the
+trie is unspecified, so rows are compared after sorting.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from inputs import (er_graph, rmat_graph, grid_graph, complete_graph, cycle_graph, star_graph,
+                    graph_from_edges, named_query, query_from_edges, DENSE5, SPARSE5, dense_family)
+
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def cuts():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_xiangkshs21_b200 import Cuts
+    return Cuts
+
+
+@pytest.fixture(scope="module")
+def ctx(cuts):
+    return cuts(device=0, arena_bytes=1 << 30)
+
+
+def _set(ctx, q, order=None):
+    qr, qc = q.csr()
+    ctx.set_query(qr, qc, order)
+
+
+def _sorted_rows(t):
+    a = t.cpu().numpy().view(np.uint32)
+    if a.size == 0:
+        return a.reshape(0, t.shape[1] if t.dim() == 2 else 0)
+    return a[np.lexsort(a.T[::-1])]
+
+
+def _check_full(ctx, g, q, enumerate_=True, modes=("bfs", "hybrid")):
+    want, lv = oracle.count(g, q, levels=True)
+    _set(ctx, q)
+    for mode in modes:
+        got = ctx.count(mode)
+        assert got == want, (g.name, q.name, mode, got, want)
+        st = ctx.stats()
+        assert st["level_size"] == lv, (g.name, q.name, mode, st["level_size"], lv)
+        assert st["order"] == oracle.order(q)
+    if enumerate_:
+        rows = ctx.enumerate("hybrid", cap_rows=want)
+        assert np.array_equal(_sorted_rows(rows), oracle.enumerate_rows(g, q)), (g.name, q.name)
+
+
+# ----------------------------------------------------------------- C1 config
+@pytest.mark.parametrize("seed", [1, 2, 3, 4, 5])
+def test_c1_er1000_triangle_c4(ctx, seed):
+    """BASELINE configs[0]: K3 and C4 on ER G(1000, 4000), count + levels + sorted rows."""
+    g = er_graph(1000, 4000, seed)
+    ctx.load_csr(g, validate=True)
+    for q in (named_query("K3"), named_query("C4")):
+        _check_full(ctx, g, q)
+
+
+def test_c1_tiny_arena_hybrid_and_bfs_enomem(cuts):
+    """Fault injection: a 64 KiB arena forces many hybrid chunks;
+    BFS must report CUTS_ENOMEM where a level does not fit."""
+    from paper_conf_sc_xiangkshs21_b200 import CutsError
+    g = er_graph(1000, 4000, 1)
+    small = cuts(device=0, arena_bytes=64 << 10)
+    small.load_csr(g)
+    q = named_query("C4")
+    want, lv = oracle.count(g, q, levels=True)
+    _set(small, q)
+    assert small.count("hybrid") == want
+    st = small.stats()
+    assert st["level_size"] == lv and st["chunks"] > 10
+    with pytest.raises(CutsError) as ei:
+        small.count("bfs")
+    assert ei.value.status == -2
+
+
+@pytest.mark.parametrize("arena_kib", [64, 96, 256, 1024])
+def test_chunk_invariance(cuts, arena_kib):
+    g = rmat_graph(9, 4, seed=2)
+    c = cuts(device=0, arena_bytes=arena_kib << 10)
+    c.load_csr(g)
+    for q in (DENSE5[9], SPARSE5[3], named_query("C4")):
+        want, lv = oracle.count(g, q, levels=True)
+        _set(c, q)
+        assert c.count("hybrid") == want, (arena_kib, q.name)
+        assert c.stats()["level_size"] == lv
+
+
+# ------------------------------------------------------------ 5-vertex family
+@pytest.mark.parametrize("seed", [2, 3])
+def test_5vertex_families_rmat9(ctx, seed):
+    g = rmat_graph(9, 4, seed=seed)
+    ctx.load_csr(g)
+    for q in DENSE5 + SPARSE5:
+        want, lv = oracle.count(g, q, levels=True)
+        _set(ctx, q)
+        for mode in ("bfs", "hybrid"):
+            assert ctx.count(mode) == want, (q.name, mode)
+            assert ctx.stats()["level_size"] == lv, (q.name, mode)
+
+
+def test_5vertex_enumerate_er(ctx):
+    g = er_graph(120, 900, 3)
+    ctx.load_csr(g)
+    for q in DENSE5 + SPARSE5:
+        _check_full(ctx, g, q, modes=("hybrid",))
+
+
+def test_dense_6_7_8_families(ctx):
+    g = er_graph(26, 230, 5)
+    ctx.load_csr(g)
+    for k in (6, 7, 8):
+        for q in dense_family(k):
+            want, lv = oracle.count(g, q, levels=True)
+            _set(ctx, q)
+            assert ctx.count("hybrid") == want, q.name
+            assert ctx.stats()["level_size"] == lv, q.name
+            assert ctx.count("bfs") == want, q.name
+
+
+def test_dense8_enumerate(ctx):
+    g = complete_graph(10)
+    ctx.load_csr(g)
+    for q in dense_family(8)[::3]:
+        _check_full(ctx, g, q, modes=("hybrid",))
+
+
+# ------------------------------------------------------------------ structure
+def test_closed_forms_on_gpu(ctx):
+    g = grid_graph(4, 4)
+    ctx.load_csr(g)
+    _set(ctx, named_query("P4"))
+    assert ctx.count("bfs") == 232
+    assert ctx.stats()["level_size"][1:3] == [16, 48]       # Fig. 2
+    g = cycle_graph(9)
+    ctx.load_csr(g)
+    for k in range(3, 9):
+        _set(ctx, named_query(f"C{k}"))
+        assert ctx.count("hybrid") == (18 if k == 9 else 0)
+        _set(ctx, named_query(f"P{k}"))
+        assert ctx.count("hybrid") == 18
+    g = er_graph(500, 3000, 7)
+    ctx.load_csr(g)
+    d = g.degrees()
+    for s in (1, 2, 3, 4):
+        _set(ctx, named_query(f"S{s}"))
+        want = sum(int(np.prod([int(x) - i for i in range(s)])) for x in d)
+        assert ctx.count("hybrid") == want
+
+
+def test_order_invariance_gpu(ctx):
+    g = er_graph(80, 500, 4)
+    ctx.load_csr(g)
+    q = DENSE5[5]
+    want = oracle.count(g, q)
+    qr, qc = q.csr()
+    import itertools
+    qe = {(u, v) for u, v in q.edges} | {(v, u) for u, v in q.edges}
+    valid = [list(p) for p in itertools.permutations(range(q.k))
+             if all(any((p[i], p[j]) in qe for j in range(i)) for i in range(1, q.k))]
+    assert len(valid) > 20
+    for o in valid[::len(valid) // 6]:
+        ctx.set_query(qr, qc, o)
+        assert ctx.count("hybrid") == want
+        _, lv = oracle.count(g, q, order=o, levels=True)
+        assert ctx.stats()["level_size"] == lv
+
+
+def test_root_range_and_slices(ctx):
+    g = rmat_graph(9, 4, seed=5)
+    ctx.load_csr(g)
+    q = DENSE5[8]
+    _set(ctx, q)
+    total = ctx.count("hybrid")
+    assert total == oracle.count(g, q)
+    l1 = ctx.stats()["level1_canonical"]
+    cuts_ = [0, 7, 40, 41, l1 // 2, l1]
+    for a, b in zip(cuts_, cuts_[1:]):
+        ctx.set_root_range(a, b)
+        assert ctx.count("hybrid") == oracle.count(g, q, root_begin=a, root_end=b)
+    ctx.set_root_range()
+    for nparts in (2, 3, 8):
+        s = 0
+        for p in range(nparts):
+            ctx.set_root_slice(0, 2**64 - 1, p, nparts)
+            s += ctx.count("hybrid")
+        assert s == total
+    # contiguous chunks of the shuffled list (the dynamic root-queue unit)
+    s = 0
+    for b in range(0, l1, 13):
+        ctx.set_root_slice(b, b + 13, 0, 1)
+        s += ctx.count("bfs")
+    assert s == total
+
+
+def test_edge_cases(ctx):
+    from paper_conf_sc_xiangkshs21_b200 import CutsError
+    # k = 1 and k = 2
+    g = er_graph(50, 120, 1)
+    ctx.load_csr(g)
+    _set(ctx, named_query("K1"))
+    assert ctx.count("bfs") == 50
+    rows = ctx.enumerate("hybrid", cap_rows=50)
+    assert sorted(rows.cpu().numpy().ravel().tolist()) == list(range(50))
+    _set(ctx, named_query("P2"))
+    assert ctx.count("hybrid") == 240
+    # graph without edges, isolated vertices
+    e = graph_from_edges(10, [])
+    ctx.load_csr(e)
+    _set(ctx, named_query("K3"))
+    assert ctx.count("hybrid") == 0 and ctx.count("bfs") == 0
+    _set(ctx, named_query("K1"))
+    assert ctx.count("hybrid") == 10
+    # query larger than any possible match
+    ctx.load_csr(star_graph(5))
+    _set(ctx, named_query("K3"))
+    assert ctx.count("hybrid") == 0
+    _set(ctx, named_query("S5"))
+    assert ctx.count("hybrid") == 120
+    # truncated enumeration reports the exact count
+    g = complete_graph(6)
+    ctx.load_csr(g)
+    _set(ctx, named_query("K3"))
+    rows = ctx.enumerate("bfs", cap_rows=10)
+    assert ctx.truncated and rows.shape[0] == 10 and ctx.stats()["count"] == 120
+    # disconnected query / bad order / bad graph
+    with pytest.raises(CutsError) as ei:
+        ctx.set_query_edges(4, [(0, 1), (2, 3)])
+    assert ei.value.status == -7
+    with pytest.raises(CutsError) as ei:
+        qr, qc = named_query("P4").csr()
+        ctx.set_query(qr, qc, [0, 2, 1, 3])
+    assert ei.value.status == -1
+    from inputs import CSRGraph
+    bad = CSRGraph(n=3, row_ptr=np.array([0, 1, 1, 1], np.uint64), col=np.array([1], np.uint32))
+    with pytest.raises(CutsError):
+        ctx.load_csr(bad, validate=True)
+    bad = CSRGraph(n=3, row_ptr=np.array([0, 2, 3, 4], np.uint64), col=np.array([2, 1, 0, 0], np.uint32))
+    with pytest.raises(CutsError):
+        ctx.load_csr(bad, validate=True)
+
+
+def test_state_errors(cuts):
+    from paper_conf_sc_xiangkshs21_b200 import CutsError
+    c = cuts(device=0, arena_bytes=1 << 20)
+    with pytest.raises(CutsError) as ei:
+        c.count("bfs")
+    assert ei.value.status == -6
+
+
+def test_fig3_trie_decode_gpu(ctx):
+    """Fig. 3: GPU decode of the paper's (CA, PA) trie == oracle decode."""
+    fx = json.load(open(os.path.join(GOLDEN, "fig3_trie.json")))
+    got = ctx.trie_decode(fx["cuts_CA"], fx["cuts_PA"]).cpu().numpy()
+    want = oracle.trie_decode(fx["cuts_CA"], fx["cuts_PA"])
+    assert np.array_equal(got.view(np.uint32), want)
+
+
+def test_alg_bytes_instrumentation(ctx):
+    """Instrumented run: the §8.d byte model is counted and timing is recorded."""
+    g = rmat_graph(9, 4, seed=2)
+    ctx.load_csr(g)
+    _set(ctx, DENSE5[0])
+    ctx.set_debug(timing=True, bytes_=True)
+    c = ctx.count("hybrid")
+    st = ctx.stats()
+    ctx.set_debug()
+    assert c == oracle.count(g, DENSE5[0])
+    assert st["alg_bytes_extend"] > 0 and st["alg_bytes_plan"] > 0
+    assert st["ms_extend"] > 0 and st["extend_launches"] >= 1
