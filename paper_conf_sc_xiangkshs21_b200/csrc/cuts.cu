@@ -235,17 +235,30 @@ void launch_plan(cuts_ctx* ctx, int J, const Graph& g, const Trie& t, const Wind
     }
 }
 
+template <int J, int M, int G>
+void launch_extend_g(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
+                     uint2* out_level, uint32_t* out_rows, uint64_t cap) {
+    static int occ = 0;
+    if (!occ) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<J, M, G>, 256, 0);
+        if (occ < 1) occ = 1;
+    }
+    // persistent-style grid: every resident CTA slot, entries fetched dynamically
+    uint64_t need = ((t1 - t0) + 255) / 256 + 1;
+    uint64_t grid = std::min<uint64_t>((uint64_t)ctx->num_sms * occ, std::max<uint64_t>(need, 1));
+    k_extend<J, M, G><<<(unsigned)grid, 256, 0, ctx->stream>>>(g, ctx->q, w.w0, w.W, w.path, w.src, w.offs, t0, t1,
+                                                               out_level, out_rows, cap, ctx->ctrl,
+                                                               (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0);
+}
+
 template <int J, int M>
 void launch_extend_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
-    uint64_t tiles = (t1 - t0 + kTile - 1) / kTile;
-    int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<J, M>, kTile, 0);
-    if (occ < 1) occ = 1;
-    uint64_t grid = std::min<uint64_t>(tiles, (uint64_t)ctx->num_sms * occ * 4);
-    k_extend<J, M><<<(unsigned)grid, kTile, 0, ctx->stream>>>(g, ctx->q, w.w0, w.W, w.path, w.src, w.offs, t0, t1,
-                                                              out_level, out_rows, cap, ctx->ctrl,
-                                                              (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0);
+    // virtual-warp width from the average candidate-list length
+    const double avg = (double)w.total / (double)std::max<uint32_t>(w.W, 1);
+    if (avg >= 40) launch_extend_g<J, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else if (avg >= 12) launch_extend_g<J, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else launch_extend_g<J, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
 }
 
 template <int M>
@@ -308,6 +321,7 @@ cuts_status extend_range(cuts_ctx* ctx, Run& r, int J, const Window& w, uint64_t
                          uint2* out, uint64_t cap) {
     if (t1 <= t0) return CUTS_OK;
     int e0 = -1;
+    CK(cudaMemsetAsync(ctx->ctrl + kWork, 0, sizeof(unsigned long long), ctx->stream));
     if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
     if (mode == kWrite) launch_extend_m<kWrite>(ctx, J, r.g, w, t0, t1, out, nullptr, cap);
     else if (mode == kCount) launch_extend_m<kCount>(ctx, J, r.g, w, t0, t1, nullptr, nullptr, 0);

@@ -45,7 +45,7 @@ enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 
 // control block (u64 words in the arena)
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
-            kEnumCursor = 6, kNumSel = 7, kCtrlWords = 64 };
+            kEnumCursor = 6, kNumSel = 7, kWork = 8, kCtrlWords = 64 };
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
     if (v == 0) return;
@@ -198,107 +198,184 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
 }
 
 // ---------------------------------------------------------------- extend
-// Items [t0, t1) of the window's flat candidate space (offs = exclusive scan of
-// ub, W+1 entries).  J = matched positions of the parents; the child takes
-// position J.  M selects the output: kWrite -> level J+1 entries (vertex,
-// parent = w0 + e) at ctrl[kCursor] (dropped past cap; the caller sizes cap so
-// that never happens in HYBRID); kCount -> 128-bit count; kEnum -> rows of k u32
-// in query-id order at ctrl[kEnumCursor].
-template <int J, int M>
-__global__ void __launch_bounds__(kTile) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
-                                                  const uint32_t* __restrict__ path_s,
-                                                  const uint64_t* __restrict__ src_off,
-                                                  const uint64_t* __restrict__ offs,
-                                                  uint64_t t0, uint64_t t1,
-                                                  uint2* __restrict__ out_level,
-                                                  uint32_t* __restrict__ out_rows, uint64_t cap,
-                                                  unsigned long long* __restrict__ ctrl, int count_bytes) {
-    __shared__ uint64_t s_offs[kTile + 1];
-    __shared__ uint32_t s_ef;
-    const uint32_t bw = q.bw[J];
-    const uint32_t qd = q.qdeg[J];
-    const int lane = threadIdx.x & 31;
-    unsigned long long my_count = 0, bytes = 0;
+// lower bound of c in sorted col[b, e): first position p with col[p] >= c
+__device__ __forceinline__ uint64_t lower_bound_u32(const uint32_t* __restrict__ col, uint64_t b, uint64_t e,
+                                                    uint32_t c) {
+    uint64_t len = e - b;
+    const uint32_t* base = col + b;
+    while (len > 0) {
+        uint64_t half = len >> 1;
+        if (__ldg(base + half) < c) { base += half + 1; len -= half + 1; }
+        else len = half;
+    }
+    return (uint64_t)(base - col);
+}
 
-    for (uint64_t base = t0 + (uint64_t)blockIdx.x * kTile; base < t1; base += (uint64_t)gridDim.x * kTile) {
-        if (threadIdx.x == 0) {          // last entry e with offs[e] <= base
+constexpr int kBatch = 4;   // entries grabbed per virtual warp per atomic
+
+// Items [t0, t1) of the window's flat candidate space (offs = exclusive scan of
+// ub, W+1 entries, ub(e) = |source list|).  J = matched positions of the
+// parents; the child takes position J.
+//
+// Mapping: a virtual warp of G lanes per entry (the paper's single-bin virtual
+// warps sized from the average degree), entries fetched dynamically
+// in batches.  Per entry the path and the backward lists' bounds are loaded
+// once into registers (uniform across the virtual warp); the G lanes walk the
+// source list G candidates at a time (coalesced), apply injectivity and the
+// degree filter, then test membership in the other backward lists, shortest
+// first, each by a binary search that starts at a per-list cursor which only
+// moves forward (candidates arrive in ascending order).  Output: one ballot per
+// warp and one atomic per warp per chunk.
+//
+// M: kWrite -> level J+1 entries (vertex, parent = w0 + e) at ctrl[kCursor]
+// (dropped past cap; HYBRID sizes cap so that never happens); kCount -> 128-bit
+// count; kEnum -> rows of k u32 in query-id order at ctrl[kEnumCursor].
+template <int J, int M, int G>
+__global__ void __launch_bounds__(256) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
+                                               const uint32_t* __restrict__ path_s,
+                                               const uint64_t* __restrict__ src_off,
+                                               const uint64_t* __restrict__ offs,
+                                               uint64_t t0, uint64_t t1,
+                                               uint2* __restrict__ out_level,
+                                               uint32_t* __restrict__ out_rows, uint64_t cap,
+                                               unsigned long long* __restrict__ ctrl, int count_bytes) {
+    constexpr int VPW = 32 / G;
+    __shared__ uint32_t s_ent[2];
+    if (threadIdx.x == 0) {        // entries holding items t0 and t1-1
+        uint64_t tt[2] = {t0, t1 - 1};
+        for (int z = 0; z < 2; ++z) {
             uint32_t lo = 0, hi = W - 1;
             while (lo < hi) {
                 uint32_t mid = (lo + hi + 1) >> 1;
-                if (offs[mid] <= base) lo = mid; else hi = mid - 1;
+                if (offs[mid] <= tt[z]) lo = mid; else hi = mid - 1;
             }
-            s_ef = lo;
+            s_ent[z] = lo;
         }
-        __syncthreads();
-        const uint32_t ef = s_ef;
-        for (int x = threadIdx.x; x <= kTile; x += blockDim.x) {
-            uint64_t e = (uint64_t)ef + x;
-            s_offs[x] = e <= W ? offs[e] : ~0ull;
-        }
-        __syncthreads();
+    }
+    __syncthreads();
+    const uint32_t ea = s_ent[0];
+    const uint32_t nent = s_ent[1] - ea + 1;
+    const int lane = threadIdx.x & 31;
+    const int vl = lane & (G - 1);
+    const int vb = lane & ~(G - 1);
+    const uint32_t bw = q.bw[J];
+    const uint32_t qd = q.qdeg[J];
+    unsigned long long my_count = 0, bytes = 0;
+    unsigned int* work = (unsigned int*)(ctrl + kWork);
 
-        const uint64_t t = base + threadIdx.x;
-        bool ok = false;
-        uint32_t c = 0, e = 0;
-        uint32_t path[J];
-        if (t < t1) {
-            uint64_t start;
-            if (s_offs[kTile] > t) {     // entries have ub >= 1, so the tile's entries fit in smem
-                int lo = 0, hi = kTile - 1;
-                while (lo < hi) {
-                    int mid = (lo + hi + 1) >> 1;
-                    if (s_offs[mid] <= t) lo = mid; else hi = mid - 1;
-                }
-                e = ef + lo;
-                start = s_offs[lo];
-            } else {                      // defensive: global search
-                uint32_t lo = ef, hi = W - 1;
-                while (lo < hi) {
-                    uint32_t mid = (lo + hi + 1) >> 1;
-                    if (offs[mid] <= t) lo = mid; else hi = mid - 1;
-                }
-                e = lo;
-                start = offs[lo];
+    for (;;) {
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(work, (unsigned)(VPW * kBatch));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (base >= nent) break;
+#pragma unroll 1
+        for (int bt = 0; bt < kBatch; ++bt) {
+            const uint32_t ei = base + (uint32_t)(bt * VPW + lane / G);
+            if (!__any_sync(0xffffffffu, ei < nent)) break;
+            const bool has = ei < nent;
+            const uint32_t e = ea + (has ? ei : 0);
+            // this entry's item range, clipped to [t0, t1)
+            uint64_t lo = 0, hi = 0;
+            if (has) {
+                const uint64_t o0 = offs[e], o1 = offs[e + 1];
+                lo = (o0 > t0 ? o0 : t0) - o0;
+                hi = (o1 < t1 ? o1 : t1) - o0;
             }
-            const uint64_t so = src_off[e];
-            c = g.col[so + (t - start)];
+            const uint64_t so = has ? src_off[e] : 0;
+            uint32_t path[J];
 #pragma unroll
-            for (int p = 0; p < J; ++p) path[p] = path_s[(size_t)p * W + e];
-            bool inj = true;
+            for (int p = 0; p < J; ++p) path[p] = has ? path_s[(size_t)p * W + e] : 0xffffffffu;
+            // other backward lists (all but the source), sorted by length ascending;
+            // fixed register slots (compile-time indices), unused slots sort last
+            uint64_t lb[J], le[J], key[J];
+            int nl = 0;
 #pragma unroll
-            for (int p = 0; p < J; ++p) inj = inj && (path[p] != c);         // injectivity
-            bool inter = inj || count_bytes;
-#pragma unroll
-            for (int p = 0; p < J; ++p) {                                     // c-intersection (Alg. 2)
-                if (((bw >> p) & 1u) && inter) {
-                    uint64_t b = g.row_ptr[path[p]];
-                    if (b != so) inter = list_contains(g.col, b, g.row_ptr[path[p] + 1], c);
+            for (int p = 0; p < J; ++p) {
+                lb[p] = le[p] = 0;
+                key[p] = ~0ull;
+                if (((bw >> p) & 1u) && has) {
+                    const uint64_t b = g.row_ptr[path[p]];
+                    if (b != so) {
+                        lb[p] = b;
+                        le[p] = g.row_ptr[path[p] + 1];
+                        key[p] = le[p] - b;
+                        ++nl;
+                    }
                 }
             }
-            ok = inj && inter && (g.deg[c] >= qd);                            // degree filter (Def. 5)
-            if (count_bytes) bytes += (inter ? 4ull : 0ull) + (ok && M != kCount ? (M == kEnum ? 4ull * q.k : 8ull) : 0ull);
-        }
-        if (M == kCount) {
-            my_count += ok ? 1 : 0;
-        } else {
-            const unsigned m = __ballot_sync(0xffffffffu, ok);
-            const int nsel = __popc(m);
-            unsigned long long pos0 = 0;
-            if (lane == 0 && nsel) pos0 = atomicAdd(ctrl + (M == kWrite ? kCursor : kEnumCursor), (unsigned long long)nsel);
-            pos0 = __shfl_sync(0xffffffffu, pos0, 0);
-            const unsigned long long pos = pos0 + __popc(m & ((1u << lane) - 1u));
-            if (ok && pos < cap) {
-                if (M == kWrite) {
-                    out_level[pos] = make_uint2(c, (uint32_t)(w0 + e));
+#pragma unroll
+            for (int x = 0; x < J; ++x)
+#pragma unroll
+                for (int y = 0; y + 1 < J - x; ++y)
+                    if (key[y + 1] < key[y]) {
+                        uint64_t tk = key[y], tb = lb[y], te = le[y];
+                        key[y] = key[y + 1]; lb[y] = lb[y + 1]; le[y] = le[y + 1];
+                        key[y + 1] = tk; lb[y + 1] = tb; le[y + 1] = te;
+                    }
+            // warp-uniform list count: every lane must reach the ballots/shuffles below
+            int nl_w = nl;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) nl_w = max(nl_w, __shfl_xor_sync(0xffffffffu, nl_w, o));
+            // chunk loop, uniform across the warp
+            uint32_t nit = (uint32_t)((hi - lo + G - 1) / G);
+            uint32_t nit_max = nit;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
+            for (uint32_t it = 0; it < nit_max; ++it) {
+                const uint64_t i = lo + (uint64_t)it * G + vl;
+                const bool act = it < nit && i < hi;
+                const uint32_t c = act ? __ldg(g.col + so + i) : 0u;
+                bool inj = act;
+#pragma unroll
+                for (int p = 0; p < J; ++p) inj = inj && (path[p] != c);      // injectivity
+                bool ok = inj && (__ldg(g.deg + c) >= qd);                   // degree filter (Def. 5)
+                bool inter = count_bytes ? act : ok;
+#pragma unroll
+                for (int x = 0; x < J; ++x) {                                 // c-intersection (Alg. 2)
+                    if (x < nl_w) {
+                        const unsigned alive = __ballot_sync(0xffffffffu, inter && x < nl);
+                        if (alive) {
+                            uint64_t mx = lb[x];
+                            if (inter && x < nl) {
+                                const uint64_t pos = lower_bound_u32(g.col, lb[x], le[x], c);
+                                inter = pos < le[x] && __ldg(g.col + pos) == c;
+                                mx = pos;
+                            }
+                            // advance this list's cursor to the vwarp's largest lower bound:
+                            // later candidates are larger, so nothing before it can match
+#pragma unroll
+                            for (int o = G / 2; o > 0; o >>= 1) {
+                                uint64_t v = __shfl_xor_sync(0xffffffffu, mx, o);
+                                mx = v > mx ? v : mx;
+                            }
+                            if (x < nl && mx > lb[x] && mx <= le[x]) lb[x] = mx;
+                        }
+                    }
+                }
+                if (count_bytes) bytes += (inter ? 4ull : 0ull) + (inter && ok && M != kCount ? (M == kEnum ? 4ull * q.k : 8ull) : 0ull);
+                ok = ok && inter;
+                if (M == kCount) {
+                    my_count += ok ? 1 : 0;
                 } else {
-                    uint32_t* row = out_rows + pos * q.k;
+                    const unsigned m = __ballot_sync(0xffffffffu, ok);
+                    const int nsel = __popc(m);
+                    unsigned long long pos0 = 0;
+                    if (lane == 0 && nsel) pos0 = atomicAdd(ctrl + (M == kWrite ? kCursor : kEnumCursor), (unsigned long long)nsel);
+                    pos0 = __shfl_sync(0xffffffffu, pos0, 0);
+                    const unsigned long long pos = pos0 + __popc(m & ((1u << lane) - 1u));
+                    if (ok && pos < cap) {
+                        if (M == kWrite) {
+                            out_level[pos] = make_uint2(c, (uint32_t)(w0 + e));
+                        } else {
+                            uint32_t* row = out_rows + pos * q.k;
 #pragma unroll
-                    for (int p = 0; p < J; ++p) row[q.S[p]] = path[p];
-                    row[q.S[J]] = c;
+                            for (int p = 0; p < J; ++p) row[q.S[p]] = path[p];
+                            row[q.S[J]] = c;
+                        }
+                    }
                 }
             }
         }
-        __syncthreads();
     }
     if (M == kCount) {
         my_count = warp_sum(my_count);
@@ -308,6 +385,7 @@ __global__ void __launch_bounds__(kTile) k_extend(Graph g, QPlan q, uint64_t w0,
         bytes = warp_sum(bytes);
         if (lane == 0) atomicAdd(ctrl + kBytesExt, bytes);
     }
+    (void)vb;
 }
 
 // ---------------------------------------------------------------- trie decode
