@@ -231,7 +231,7 @@ constexpr int kBatch = 4;   // entries grabbed per virtual warp per atomic
 // (dropped past cap; HYBRID sizes cap so that never happens); kCount -> 128-bit
 // count; kEnum -> rows of k u32 in query-id order at ctrl[kEnumCursor].
 template <int J, int M, int G>
-__global__ void __launch_bounds__(256) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
+__global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
                                                const uint32_t* __restrict__ path_s,
                                                const uint64_t* __restrict__ src_off,
                                                const uint64_t* __restrict__ offs,
@@ -240,6 +240,7 @@ __global__ void __launch_bounds__(256) k_extend(Graph g, QPlan q, uint64_t w0, u
                                                uint32_t* __restrict__ out_rows, uint64_t cap,
                                                unsigned long long* __restrict__ ctrl, int count_bytes) {
     constexpr int VPW = 32 / G;
+    constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
     __shared__ uint32_t s_ent[2];
     if (threadIdx.x == 0) {        // entries holding items t0 and t1-1
         uint64_t tt[2] = {t0, t1 - 1};
@@ -287,18 +288,18 @@ __global__ void __launch_bounds__(256) k_extend(Graph g, QPlan q, uint64_t w0, u
             for (int p = 0; p < J; ++p) path[p] = has ? path_s[(size_t)p * W + e] : 0xffffffffu;
             // other backward lists (all but the source), sorted by length ascending;
             // fixed register slots (compile-time indices), unused slots sort last
-            uint64_t lb[J], le[J], key[J];
+            const uint32_t* lb[J];     // list cursor (advances)
+            uint32_t ln[J];            // remaining length; unused slots sort last
             int nl = 0;
 #pragma unroll
             for (int p = 0; p < J; ++p) {
-                lb[p] = le[p] = 0;
-                key[p] = ~0ull;
+                lb[p] = g.col;
+                ln[p] = 0xffffffffu;
                 if (((bw >> p) & 1u) && has) {
                     const uint64_t b = g.row_ptr[path[p]];
                     if (b != so) {
-                        lb[p] = b;
-                        le[p] = g.row_ptr[path[p] + 1];
-                        key[p] = le[p] - b;
+                        lb[p] = g.col + b;
+                        ln[p] = (uint32_t)(g.row_ptr[path[p] + 1] - b);
                         ++nl;
                     }
                 }
@@ -307,10 +308,11 @@ __global__ void __launch_bounds__(256) k_extend(Graph g, QPlan q, uint64_t w0, u
             for (int x = 0; x < J; ++x)
 #pragma unroll
                 for (int y = 0; y + 1 < J - x; ++y)
-                    if (key[y + 1] < key[y]) {
-                        uint64_t tk = key[y], tb = lb[y], te = le[y];
-                        key[y] = key[y + 1]; lb[y] = lb[y + 1]; le[y] = le[y + 1];
-                        key[y + 1] = tk; lb[y + 1] = tb; le[y + 1] = te;
+                    if (ln[y + 1] < ln[y]) {
+                        const uint32_t tl = ln[y];
+                        const uint32_t* tb = lb[y];
+                        ln[y] = ln[y + 1]; lb[y] = lb[y + 1];
+                        ln[y + 1] = tl; lb[y + 1] = tb;
                     }
             // warp-uniform list count: every lane must reach the ballots/shuffles below
             int nl_w = nl;
@@ -328,27 +330,33 @@ __global__ void __launch_bounds__(256) k_extend(Graph g, QPlan q, uint64_t w0, u
                 bool inj = act;
 #pragma unroll
                 for (int p = 0; p < J; ++p) inj = inj && (path[p] != c);      // injectivity
-                bool ok = inj && (__ldg(g.deg + c) >= qd);                   // degree filter (Def. 5)
+                bool ok = inj && (qd <= 1 || __ldg(g.deg + c) >= qd);       // degree filter (Def. 5);
+                                                                              // every neighbour has deg >= 1
                 bool inter = count_bytes ? act : ok;
 #pragma unroll
                 for (int x = 0; x < J; ++x) {                                 // c-intersection (Alg. 2)
                     if (x < nl_w) {
-                        const unsigned alive = __ballot_sync(0xffffffffu, inter && x < nl);
-                        if (alive) {
-                            uint64_t mx = lb[x];
-                            if (inter && x < nl) {
-                                const uint64_t pos = lower_bound_u32(g.col, lb[x], le[x], c);
-                                inter = pos < le[x] && __ldg(g.col + pos) == c;
-                                mx = pos;
+                        const bool pend = inter && x < nl;
+                        const unsigned pw = __ballot_sync(0xffffffffu, pend);
+                        if (pw) {
+                            uint32_t pos = 0;
+                            if (pend) {     // branch-free lower bound from the cursor
+                                const uint32_t* b0 = lb[x];
+                                uint32_t len = ln[x];
+                                while (len > 1) {
+                                    const uint32_t half = len >> 1;
+                                    b0 = (__ldg(b0 + half - 1) < c) ? b0 + half : b0;
+                                    len -= half;
+                                }
+                                inter = len == 1 && __ldg(b0) == c;
+                                pos = (uint32_t)(b0 - lb[x]);
                             }
-                            // advance this list's cursor to the vwarp's largest lower bound:
-                            // later candidates are larger, so nothing before it can match
-#pragma unroll
-                            for (int o = G / 2; o > 0; o >>= 1) {
-                                uint64_t v = __shfl_xor_sync(0xffffffffu, mx, o);
-                                mx = v > mx ? v : mx;
-                            }
-                            if (x < nl && mx > lb[x] && mx <= le[x]) lb[x] = mx;
+                            // candidates ascend with the lane, so the highest pending lane of
+                            // the virtual warp holds the furthest safe cursor position
+                            const unsigned pv = (pw >> vb) & kGMask;
+                            const int hl = pv ? vb + 31 - __clz(pv) : lane;
+                            const uint32_t mpos = __shfl_sync(0xffffffffu, pos, hl);
+                            if (pv && x < nl) { lb[x] += mpos; ln[x] -= mpos; }
                         }
                     }
                 }
