@@ -34,6 +34,7 @@ def _args():
     ap.add_argument("--workload", default="C2")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--chunks-per-rank", type=int, default=16, help="dynamic root queue granularity (N > 1)")
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     return ap.parse_args()
 
@@ -122,26 +123,48 @@ def run_ours(args):
         ctx.load_graph(rp, cl, validate=True)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
 
+    from paper_conf_sc_xiangkshs21_b200 import dist as D
+    store = D.default_store() if world > 1 else None
+    pass_id = [0]
+
     def set_q(c, q):
         qr, qc = q.csr()
         c.set_query(qr, qc)
-        c.set_root_slice(0, 2**64 - 1, rank, world)   # root partition across ranks
+
+    def count_q(c, q, tag):
+        """This rank's share of one query.  N = 1: all roots.  N > 1: the seeded-
+        shuffled level-1 list is cut into world*CHUNKS chunks pulled from a shared
+        atomic counter (dynamic root redistribution)."""
+        set_q(c, q)
+        if world == 1:
+            return c.count(wl.mode), [c.stats()]
+        _, l1 = c.level1_size()
+        cs = max(1, -(-l1 // (world * args.chunks_per_rank)))
+        queue = D.RootQueue(store, f"{tag}", D.n_chunks(l1, cs))
+        local, sts = 0, []
+        while (ch := queue.next()) is not None:
+            b, e = D.chunk_bounds(ch, cs)
+            c.set_root_slice(b, e, 0, 1)
+            local += c.count(wl.mode)
+            sts.append(c.stats())
+        return local, sts
 
     def step(timing=False):
         """One pass over every (graph, query); returns (local count, launches, ms_extend, launches_ext)."""
         total, launches, ms_ext, n_ext = 0, 0, 0.0, 0
         c = ctx
         c.set_debug(timing=timing)
-        for (rp, cl), (g, qs) in zip(dev_graphs, graphs):
+        pass_id[0] += 1
+        for gi, ((rp, cl), (g, qs)) in enumerate(zip(dev_graphs, graphs)):
             c.load_graph(rp, cl)                      # borrows the resident CSR, derives deg
             launches += 1
-            for q in qs:
-                set_q(c, q)
-                total += c.count(wl.mode)
-                st = c.stats()
-                launches += st["launches"]
-                ms_ext += st["ms_extend"]
-                n_ext += st["extend_launches"]
+            for qi, q in enumerate(qs):
+                cnt, sts = count_q(c, q, f"p{pass_id[0]}g{gi}q{qi}")
+                total += cnt
+                for st in sts:
+                    launches += st["launches"]
+                    ms_ext += st["ms_extend"]
+                    n_ext += st["extend_launches"]
         return total, launches, ms_ext, n_ext
 
     def barrier():
@@ -174,17 +197,8 @@ def run_ours(args):
     step_ms_local = sum(times) / len(times)
     local_count = counts[-1]
     # exchange: sum of counts over ranks, max of time over ranks
-    if world > 1:
-        import torch.distributed as dist
-        t = torch.tensor([step_ms_local], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        step_ms = float(t.item())
-        lo_hi = torch.tensor([local_count & 0xFFFFFFFF, local_count >> 32], dtype=torch.int64, device=dev)
-        dist.all_reduce(lo_hi)
-        step_count = int(lo_hi[0].item()) + (int(lo_hi[1].item()) << 32)
-    else:
-        step_ms = step_ms_local
-        step_count = local_count
+    step_ms = D.allreduce_max(step_ms_local, device=dev)         # max over ranks
+    step_count = D.allreduce_count(local_count, device=dev)      # the one exchange: NCCL sum of counts
     value = step_count / (step_ms / 1e3)
 
     # e2e: the user's call with HOST buffers (pinned H2D of the graphs each step, counts back to host)
@@ -202,18 +216,13 @@ def run_ours(args):
                 dcl = hcl.to(dev, non_blocking=True)
                 h2d += hrp.numel() * 8 + hcl.numel() * 4
                 c.load_graph(drp, dcl)
-                for q in qs:
-                    set_q(c, q)
-                    cnt += c.count(wl.mode)
+                for qi, q in enumerate(qs):
+                    pass_id[0] += 1
+                    cnt += count_q(c, q, f"e{pass_id[0]}q{qi}")[0]
         ev1.record(stream)
         torch.cuda.synchronize(dev)
         e2e_ms.append(ev0.elapsed_time(ev1))
-    e2e_local = sum(e2e_ms) / len(e2e_ms)
-    if world > 1:
-        import torch.distributed as dist
-        t = torch.tensor([e2e_local], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_local = float(t.item())
+    e2e_local = D.allreduce_max(sum(e2e_ms) / len(e2e_ms), device=dev)
     nq = sum(len(qs) for _, qs in graphs)
 
     # algorithmic bytes of the dominant kernel (k_extend), instrumented untimed pass
@@ -221,10 +230,9 @@ def run_ours(args):
     ctx.set_debug(bytes_=True)
     for (rp, cl), (g, qs) in zip(dev_graphs, graphs):
         ctx.load_graph(rp, cl)
-        for q in qs:
-            set_q(ctx, q)
-            ctx.count(wl.mode)
-            alg_ext += ctx.stats()["alg_bytes_extend"]
+        for qi, q in enumerate(qs):
+            pass_id[0] += 1
+            alg_ext += sum(st["alg_bytes_extend"] for st in count_q(ctx, q, f"b{pass_id[0]}q{qi}")[1])
     ctx.set_debug()
     peak, peak_src = _peaks()
     per_step_ext_ms = ms_ext / args.steps
@@ -244,7 +252,7 @@ def run_ours(args):
         "config": {"workload": wl.name, "description": wl.description, "queries": nq,
                    "graphs": [s.name for s, _ in wl.parts], "embeddings_per_step": step_count,
                    "mode": wl.mode, "l2": "flushed between timed steps (256 MiB write)",
-                   "parallelism": f"root-partition x{world} + NCCL all-reduce of counts"},
+                   "parallelism": (f"dynamic root-chunk queue x{world} ({args.chunks_per_rank} chunks/rank/query) + NCCL all-reduce of counts" if world > 1 else "1 GPU")},
         "e2e": {"value": step_count / (e2e_local / 1e3), "unit": "embeddings/s", "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": 8 * nq, "ms_per_step": e2e_local},
         "gpu_launches": launches // args.steps,

@@ -86,6 +86,8 @@ typedef struct {
     uint64_t alg_bytes_extend;         /* algorithmic bytes of the extend kernels (SURVEY
                                           §8.d model; only with CUTS_DEBUG_BYTES)           */
     uint64_t alg_bytes_plan;           /* algorithmic bytes of the plan kernels (ditto)     */
+    uint64_t hubs;                     /* vertices with an adjacency bitmap (see below)     */
+    uint64_t hub_threshold;            /* degree threshold used for the bitmaps             */
 } cuts_stats;
 
 /* debug / instrumentation flags for cuts_set_debug */
@@ -113,6 +115,14 @@ int cuts_version(void);
 cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz,
                             const uint64_t* d_row_ptr, const uint32_t* d_col, int validate);
 
+/* Membership rows for hub vertices (SV-style intersection, Alg. 2 l.7-17,
+ * P:1055-1072): at the next cuts_load_graph, every vertex with deg >= t gets a
+ * bitmap of its neighbours over [0, n) in the arena, and a membership test
+ * against its list becomes one load.  t = 0: automatic (the smallest power of
+ * two >= 256 whose bitmaps fit min(arena/16, 8 GiB)); t = UINT32_MAX: off.
+ * Never changes a result.  Default 0. */
+cuts_status cuts_set_hub_threshold(cuts_ctx* ctx, uint32_t t);
+
 /* Query Q as HOST CSR over 0..k-1 (1 <= k <= 8): row_ptr u32[k+1], col u32[...],
  * symmetric, no loops/duplicates, connected (else CUTS_EUNSUPPORTED).
  * order == NULL -> the paper's rule: root = max degree (ties: min id),
@@ -134,6 +144,13 @@ cuts_status cuts_set_root_range(cuts_ctx* ctx, uint64_t begin, uint64_t end);
  * root-chunk queue.  Default: begin = 0, end = UINT64_MAX, part = 0, nparts = 1. */
 cuts_status cuts_set_root_slice(cuts_ctx* ctx, uint64_t begin, uint64_t end,
                                 uint32_t part, uint32_t nparts);
+
+/* Size of the level-1 candidate list for the current query (runs the device
+ * degree-filter compaction, Alg. 1 l.8-11): *canonical = |{u : deg(u) >=
+ * deg_Q(S[0])}|, *in_range = how many of those lie in the root range (the
+ * length of the shuffled list that cuts_set_root_slice positions index).
+ * Either pointer may be NULL. */
+cuts_status cuts_level1_size(cuts_ctx* ctx, uint64_t* canonical, uint64_t* in_range);
 
 /* Exact number of ordered non-induced embeddings of Q in D restricted to the
  * selected roots.  *out = low 64 bits; CUTS_EOVERFLOW if the count is >= 2^64

@@ -22,8 +22,8 @@ MAX_K = 8
 
 # the symbols include/cuts.h declares (tests check the library exports all of them)
 EXPORTED = ["cuts_version", "cuts_create", "cuts_destroy", "cuts_last_error", "cuts_load_graph",
-            "cuts_set_query", "cuts_set_root_range", "cuts_set_root_slice", "cuts_count",
-            "cuts_enumerate", "cuts_get_stats", "cuts_set_debug", "cuts_trie_decode"]
+            "cuts_set_query", "cuts_set_root_range", "cuts_set_root_slice", "cuts_level1_size", "cuts_count",
+            "cuts_enumerate", "cuts_get_stats", "cuts_set_debug", "cuts_trie_decode", "cuts_set_hub_threshold"]
 
 
 class cuts_opts(ctypes.Structure):
@@ -40,7 +40,8 @@ class cuts_stats(ctypes.Structure):
                 ("peak_arena_bytes", ctypes.c_uint64), ("items", ctypes.c_uint64),
                 ("ms_total", ctypes.c_double), ("ms_extend", ctypes.c_double), ("ms_plan", ctypes.c_double),
                 ("extend_launches", ctypes.c_uint64), ("alg_bytes_extend", ctypes.c_uint64),
-                ("alg_bytes_plan", ctypes.c_uint64)]
+                ("alg_bytes_plan", ctypes.c_uint64), ("hubs", ctypes.c_uint64),
+                ("hub_threshold", ctypes.c_uint64)]
 
 
 _lib = None
@@ -65,10 +66,12 @@ def load() -> ctypes.CDLL:
         "cuts_set_query": ([P, u32, u32p, u32p, u32p], i32),
         "cuts_set_root_range": ([P, u64, u64], i32),
         "cuts_set_root_slice": ([P, u64, u64, u32, u32], i32),
+        "cuts_level1_size": ([P, u64p, u64p], i32),
         "cuts_count": ([P, i32, u64p], i32),
         "cuts_enumerate": ([P, i32, P, u64, u64p], i32),
         "cuts_get_stats": ([P, ctypes.POINTER(cuts_stats)], i32),
         "cuts_set_debug": ([P, u32], i32),
+        "cuts_set_hub_threshold": ([P, u32], i32),
         "cuts_trie_decode": ([P, u32, u64p, ctypes.POINTER(P), ctypes.POINTER(P), P], i32),
     }
     for name, (args, res) in sig.items():

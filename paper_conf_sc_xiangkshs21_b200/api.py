@@ -138,6 +138,17 @@ class Cuts:
         self._check(self.lib.cuts_set_root_slice(self.h, begin, end, part, nparts))
         return self
 
+    def set_hub_threshold(self, t: int | None):
+        """Bitmap rows for vertices with deg >= t at the next load (None: off, 0: auto)."""
+        self._check(self.lib.cuts_set_hub_threshold(self.h, 0xFFFFFFFF if t is None else int(t)))
+        return self
+
+    def level1_size(self):
+        """(canonical level-1 size, size inside the root range) for the current query."""
+        a, b = ctypes.c_uint64(), ctypes.c_uint64()
+        self._check(self.lib.cuts_level1_size(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return int(a.value), int(b.value)
+
     def set_debug(self, timing: bool = False, bytes_: bool = False):
         flags = (L.CUTS_DEBUG_TIMING if timing else 0) | (L.CUTS_DEBUG_BYTES if bytes_ else 0)
         self._check(self.lib.cuts_set_debug(self.h, flags))
@@ -177,7 +188,7 @@ class Cuts:
             "launches": s.launches, "peak_arena_bytes": s.peak_arena_bytes, "items": s.items,
             "ms_total": s.ms_total, "ms_extend": s.ms_extend, "ms_plan": s.ms_plan,
             "extend_launches": s.extend_launches, "alg_bytes_extend": s.alg_bytes_extend,
-            "alg_bytes_plan": s.alg_bytes_plan,
+            "alg_bytes_plan": s.alg_bytes_plan, "hubs": s.hubs, "hub_threshold": s.hub_threshold,
         }
 
     def trie_decode(self, ca_levels, pa_levels) -> torch.Tensor:

@@ -30,7 +30,7 @@ namespace {
 
 constexpr uint64_t kAlign = 256;
 constexpr uint64_t kCtrlBytes = 4096;
-constexpr uint64_t kMaxWindow = 1ull << 22;      // entries per plan window
+constexpr uint64_t kMaxWindow = 1ull << 24;      // entries per plan window
 constexpr uint64_t kMaxLevel = 0xFFFFFFFFull;    // u32 parent indices
 
 inline uint64_t align_up(uint64_t x) { return (x + kAlign - 1) & ~(kAlign - 1); }
@@ -54,7 +54,12 @@ struct cuts_ctx {
     const uint64_t* row_ptr = nullptr;
     const uint32_t* col = nullptr;
     uint32_t* deg = nullptr;
-    uint64_t base_off = 0;                 // first free byte after ctrl + deg
+    uint32_t* hub = nullptr;               // hub[v] -> bitmap row, or kNoHub
+    uint32_t* bm = nullptr;                // hub bitmaps
+    uint32_t words = 0;
+    uint64_t nhubs = 0, hub_t_used = 0;
+    uint32_t hub_t = 0;                    // requested threshold (0 auto, UINT32_MAX off)
+    uint64_t base_off = 0;                 // first free byte after ctrl + deg + bitmaps
     // query
     bool has_query = false;
     QPlan q{};
@@ -246,9 +251,12 @@ void launch_extend_g(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0
     // persistent-style grid: every resident CTA slot, entries fetched dynamically
     uint64_t need = ((t1 - t0) + 255) / 256 + 1;
     uint64_t grid = std::min<uint64_t>((uint64_t)ctx->num_sms * occ, std::max<uint64_t>(need, 1));
+    // entries per virtual-warp fetch: ~2K candidate items per atomic on the work counter
+    const double avg = (double)w.total / (double)std::max<uint32_t>(w.W, 1);
+    const uint32_t batch = (uint32_t)std::min(256.0, std::max(2.0, 2048.0 / std::max(avg, 1.0) / (32 / G)));
     k_extend<J, M, G><<<(unsigned)grid, 256, 0, ctx->stream>>>(g, ctx->q, w.w0, w.W, w.path, w.src, w.offs, t0, t1,
                                                                out_level, out_rows, cap, ctx->ctrl,
-                                                               (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0);
+                                                               (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0, batch);
 }
 
 template <int J, int M>
@@ -256,8 +264,8 @@ void launch_extend_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0
                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
     // virtual-warp width from the average candidate-list length
     const double avg = (double)w.total / (double)std::max<uint32_t>(w.W, 1);
-    if (avg >= 40) launch_extend_g<J, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
-    else if (avg >= 12) launch_extend_g<J, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    if (avg >= 96) launch_extend_g<J, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else if (avg >= 24) launch_extend_g<J, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
     else launch_extend_g<J, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
 }
 
@@ -458,6 +466,57 @@ cuts_status bfs_levels(cuts_ctx* ctx, Run& r, uint64_t N1) {
     return CUTS_OK;
 }
 
+// hub bitmaps (SV-style membership rows) after deg; moves base_off
+cuts_status build_hubs(cuts_ctx* ctx) {
+    ctx->nhubs = 0;
+    ctx->hub_t_used = 0;
+    ctx->hub = nullptr;
+    ctx->bm = nullptr;
+    if (ctx->hub_t == 0xFFFFFFFFu || ctx->n == 0 || ctx->nnz == 0) return CUTS_OK;
+    const uint32_t n = ctx->n;
+    ctx->words = (n + 31) / 32;
+    const uint64_t row_bytes = (uint64_t)ctx->words * 4;
+    const uint64_t budget = std::min<uint64_t>(ctx->arena_bytes / 16, 8ull << 30);
+    unsigned grid = (unsigned)std::min<uint64_t>(((uint64_t)n + 255) / 256, (uint64_t)ctx->num_sms * 8);
+    uint32_t t = ctx->hub_t;
+    CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
+    if (t == 0) {   // automatic: smallest power of two >= 256 whose rows fit the budget
+        k_hub_hist<<<grid, 256, 0, ctx->stream>>>(ctx->deg, n, ctx->ctrl + 16);
+        CK(cudaGetLastError());
+        TRY(read_ctrl(ctx));
+        t = 0;
+        for (int b = 8; b < 32; ++b) {
+            uint64_t cnt = 0;
+            for (int b2 = b; b2 < 32; ++b2) cnt += ctx->h_ctrl[16 + b2];
+            if (cnt * row_bytes <= budget) { t = 1u << b; break; }
+        }
+        if (t == 0) return CUTS_OK;
+        CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
+    }
+    const uint64_t hub_bytes = align_up((uint64_t)n * 4);
+    if (ctx->base_off + hub_bytes + (64u << 10) > ctx->arena_bytes) return CUTS_OK;   // no room: skip
+    ctx->hub = (uint32_t*)(ctx->arena + ctx->base_off);
+    k_hub_mark<<<grid, 256, 0, ctx->stream>>>(ctx->deg, n, t, ctx->hub, ctx->ctrl + kNumSel);
+    CK(cudaGetLastError());
+    TRY(read_ctrl(ctx));
+    const uint64_t nh = ctx->h_ctrl[kNumSel];
+    const uint64_t bm_bytes = align_up(nh * row_bytes);
+    if (nh == 0 || ctx->base_off + hub_bytes + bm_bytes + (64u << 10) > ctx->arena_bytes) {
+        ctx->hub = nullptr;
+        return CUTS_OK;   // nothing to do, or does not fit: binary search everywhere
+    }
+    ctx->bm = (uint32_t*)(ctx->arena + ctx->base_off + hub_bytes);
+    CK(cudaMemsetAsync(ctx->bm, 0, nh * row_bytes, ctx->stream));
+    unsigned g2 = (unsigned)std::min<uint64_t>(((uint64_t)n * 32 + 255) / 256, (uint64_t)ctx->num_sms * 16);
+    k_hub_fill<<<g2, 256, 0, ctx->stream>>>(ctx->row_ptr, ctx->col, n, ctx->hub, ctx->words, ctx->bm);
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->nhubs = nh;
+    ctx->hub_t_used = t;
+    ctx->base_off += hub_bytes + bm_bytes;
+    return CUTS_OK;
+}
+
 // level 1: canonical list -> root range -> shuffle -> slice
 cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
     const uint64_t top_save = ctx->top;
@@ -538,7 +597,7 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     r.enumerate = enumerate;
     r.rows = rows;
     r.cap_rows = cap_rows;
-    r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->n};
+    r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words};
     uint64_t n1 = 0;
     TRY(build_level1(ctx, r, &n1));
     ctx->st.level_size[1] = n1;
@@ -571,6 +630,8 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     ctx->st.alg_bytes_plan = ctx->h_ctrl[kBytesPlan];
     ctx->st.alg_bytes_extend = ctx->h_ctrl[kBytesExt];
     ctx->st.peak_arena_bytes = ctx->peak;
+    ctx->st.hubs = ctx->nhubs;
+    ctx->st.hub_threshold = ctx->hub_t_used;
     if (ctx->debug & CUTS_DEBUG_TIMING) {
         double ms = 0;
         for (auto& pr : ctx->ev_ext) {
@@ -662,14 +723,21 @@ cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint6
                                                     (unsigned long long)ends[0], (unsigned long long)ends[1], (unsigned long long)nnz);
     if (validate && n) {
         CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
-        Graph g{d_row_ptr, d_col, ctx->deg, n};
+        Graph g{d_row_ptr, d_col, ctx->deg, nullptr, nullptr, n, 0};
         unsigned grid = (unsigned)std::min<uint64_t>(((uint64_t)n * 32 + 255) / 256, (uint64_t)ctx->num_sms * 16);
         k_validate<<<grid, 256, 0, ctx->stream>>>(g, ctx->ctrl);
         CK(cudaGetLastError());
         TRY(read_ctrl(ctx));
         if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_EINVAL, "graph is not canonical symmetric CSR (sorted, no loops/dups, ids < n)");
     }
+    TRY(build_hubs(ctx));
     ctx->has_graph = true;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_hub_threshold(cuts_ctx* ctx, uint32_t t) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->hub_t = t;
     return CUTS_OK;
 }
 
@@ -709,6 +777,31 @@ cuts_status cuts_set_root_slice(cuts_ctx* ctx, uint64_t begin, uint64_t end, uin
     ctx->slice_end = end;
     ctx->part = part;
     ctx->nparts = nparts;
+    return CUTS_OK;
+}
+
+cuts_status cuts_level1_size(cuts_ctx* ctx, uint64_t* canonical, uint64_t* in_range) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (!ctx->has_graph || !ctx->has_query) return fail(ctx, CUTS_ESTATE, "load_graph and set_query must precede cuts_level1_size");
+    CK(cudaSetDevice(ctx->device));
+    ctx->bot = ctx->base_off;
+    ctx->top = ctx->arena_bytes & ~(kAlign - 1);
+    uint64_t off_canon, off_tmp;
+    TRY(alloc_top(ctx, (uint64_t)ctx->n * 4 + 4, &off_canon));
+    DegAtLeast pred{ctx->deg, ctx->q.qdeg[0]};
+    thrust::counting_iterator<uint32_t> it(0);
+    size_t tmp_bytes = 0;
+    CK(cub::DeviceSelect::If(nullptr, tmp_bytes, it, (uint32_t*)(ctx->arena + off_canon), ctx->ctrl + kNumSel,
+                             (int64_t)ctx->n, pred, ctx->stream));
+    TRY(alloc_top(ctx, tmp_bytes, &off_tmp));
+    CK(cub::DeviceSelect::If(ctx->arena + off_tmp, tmp_bytes, it, (uint32_t*)(ctx->arena + off_canon),
+                             ctx->ctrl + kNumSel, (int64_t)ctx->n, pred, ctx->stream));
+    TRY(read_ctrl(ctx));
+    const uint64_t nc = ctx->h_ctrl[kNumSel];
+    const uint64_t rb = std::min(ctx->root_begin, nc), re = std::max(rb, std::min(ctx->root_end, nc));
+    if (canonical) *canonical = nc;
+    if (in_range) *in_range = re - rb;
     return CUTS_OK;
 }
 

@@ -38,8 +38,14 @@ struct Graph {
     const uint64_t* __restrict__ row_ptr;
     const uint32_t* __restrict__ col;
     const uint32_t* __restrict__ deg;
+    const uint32_t* __restrict__ hub;   // hub[v] = row of v in bm, or kNoHub (nullptr: no bitmaps)
+    const uint32_t* __restrict__ bm;    // hub adjacency bitmaps, words u32 per row
     uint32_t n;
+    uint32_t words;
 };
+
+constexpr uint32_t kNoHub = 0xffffffffu;
+constexpr uint32_t kBmFlag = 0x80000000u;   // list-slot length flag: probe a bitmap instead
 
 enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 
@@ -77,6 +83,46 @@ __device__ __forceinline__ bool list_contains(const uint32_t* __restrict__ col, 
 __global__ void k_degree(const uint64_t* __restrict__ row_ptr, uint32_t n, uint32_t* __restrict__ deg) {
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x)
         deg[v] = (uint32_t)(row_ptr[v + 1] - row_ptr[v]);
+}
+
+// SV-style membership rows (Alg. 2 l.7-17's |V|-sized scatter vector, P:1055-1072,
+// precomputed once per hub vertex instead of per worker): for every vertex with
+// deg >= T a bitmap over [0, n); a membership test against a hub list is then
+// one load instead of a binary search.
+__global__ void k_hub_hist(const uint32_t* __restrict__ deg, uint32_t n, unsigned long long* __restrict__ hist) {
+    // hist[b] = #vertices with deg >= 2^b, b < 32
+    __shared__ unsigned int s[32];
+    if (threadIdx.x < 32) s[threadIdx.x] = 0;
+    __syncthreads();
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        const uint32_t d = deg[v];
+        if (d) atomicAdd(&s[31 - __clz(d)], 1u);
+    }
+    __syncthreads();
+    if (threadIdx.x < 32 && s[threadIdx.x]) atomicAdd(hist + threadIdx.x, (unsigned long long)s[threadIdx.x]);
+}
+
+__global__ void k_hub_mark(const uint32_t* __restrict__ deg, uint32_t n, uint32_t t, uint32_t* __restrict__ hub,
+                           unsigned long long* __restrict__ counter) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x)
+        hub[v] = deg[v] >= t ? (uint32_t)atomicAdd(counter, 1ull) : kNoHub;
+}
+
+// one warp per vertex: hubs set the bits of their neighbours
+__global__ void k_hub_fill(const uint64_t* __restrict__ row_ptr, const uint32_t* __restrict__ col, uint32_t n,
+                           const uint32_t* __restrict__ hub, uint32_t words, uint32_t* __restrict__ bm) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t v = warp; v < n; v += nwarps) {
+        const uint32_t h = hub[v];
+        if (h == kNoHub) continue;
+        uint32_t* row = bm + (uint64_t)h * words;
+        for (uint64_t p = row_ptr[v] + lane; p < row_ptr[v + 1]; p += 32) {
+            const uint32_t u = col[p];
+            atomicOr(row + (u >> 5), 1u << (u & 31));
+        }
+    }
 }
 
 // graph validation: sorted strictly ascending rows, no loops, ids < n, symmetric.
@@ -211,7 +257,6 @@ __device__ __forceinline__ uint64_t lower_bound_u32(const uint32_t* __restrict__
     return (uint64_t)(base - col);
 }
 
-constexpr int kBatch = 4;   // entries grabbed per virtual warp per atomic
 
 // Items [t0, t1) of the window's flat candidate space (offs = exclusive scan of
 // ub, W+1 entries, ub(e) = |source list|).  J = matched positions of the
@@ -238,7 +283,8 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                                                uint64_t t0, uint64_t t1,
                                                uint2* __restrict__ out_level,
                                                uint32_t* __restrict__ out_rows, uint64_t cap,
-                                               unsigned long long* __restrict__ ctrl, int count_bytes) {
+                                               unsigned long long* __restrict__ ctrl, int count_bytes,
+                                               uint32_t batch) {
     constexpr int VPW = 32 / G;
     constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
     __shared__ uint32_t s_ent[2];
@@ -261,17 +307,18 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
     const int vb = lane & ~(G - 1);
     const uint32_t bw = q.bw[J];
     const uint32_t qd = q.qdeg[J];
+    const int nl_s = __popc(bw) - 1;   // lists besides the source (same for every entry)
     unsigned long long my_count = 0, bytes = 0;
     unsigned int* work = (unsigned int*)(ctrl + kWork);
 
     for (;;) {
         uint32_t base = 0;
-        if (lane == 0) base = atomicAdd(work, (unsigned)(VPW * kBatch));
+        if (lane == 0) base = atomicAdd(work, (unsigned)VPW * batch);
         base = __shfl_sync(0xffffffffu, base, 0);
         if (base >= nent) break;
 #pragma unroll 1
-        for (int bt = 0; bt < kBatch; ++bt) {
-            const uint32_t ei = base + (uint32_t)(bt * VPW + lane / G);
+        for (uint32_t bt = 0; bt < batch; ++bt) {
+            const uint32_t ei = base + bt * VPW + (uint32_t)(lane / G);
             if (!__any_sync(0xffffffffu, ei < nent)) break;
             const bool has = ei < nent;
             const uint32_t e = ea + (has ? ei : 0);
@@ -290,39 +337,50 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
             // fixed register slots (compile-time indices), unused slots sort last
             const uint32_t* lb[J];     // list cursor (advances)
             uint32_t ln[J];            // remaining length; unused slots sort last
-            int nl = 0;
 #pragma unroll
             for (int p = 0; p < J; ++p) {
                 lb[p] = g.col;
                 ln[p] = 0xffffffffu;
-                if (((bw >> p) & 1u) && has) {
-                    const uint64_t b = g.row_ptr[path[p]];
-                    if (b != so) {
-                        lb[p] = g.col + b;
-                        ln[p] = (uint32_t)(g.row_ptr[path[p] + 1] - b);
-                        ++nl;
+            }
+            if (nl_s > 0 && has) {
+#pragma unroll
+                for (int p = 0; p < J; ++p) {
+                    if ((bw >> p) & 1u) {
+                        const uint64_t b = g.row_ptr[path[p]];
+                        if (b != so) {
+                            const uint32_t h = g.hub ? __ldg(g.hub + path[p]) : kNoHub;
+                            if (h != kNoHub) {     // hub list: probe its bitmap row (sorts last)
+                                lb[p] = g.bm + (uint64_t)h * g.words;
+                                ln[p] = kBmFlag | (uint32_t)(g.row_ptr[path[p] + 1] - b);
+                            } else {
+                                lb[p] = g.col + b;
+                                ln[p] = (uint32_t)(g.row_ptr[path[p] + 1] - b);
+                            }
+                        }
                     }
                 }
             }
+            if (nl_s > 1) {
 #pragma unroll
-            for (int x = 0; x < J; ++x)
+                for (int x = 0; x < J; ++x)
 #pragma unroll
-                for (int y = 0; y + 1 < J - x; ++y)
-                    if (ln[y + 1] < ln[y]) {
-                        const uint32_t tl = ln[y];
-                        const uint32_t* tb = lb[y];
-                        ln[y] = ln[y + 1]; lb[y] = lb[y + 1];
-                        ln[y + 1] = tl; lb[y + 1] = tb;
-                    }
-            // warp-uniform list count: every lane must reach the ballots/shuffles below
-            int nl_w = nl;
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) nl_w = max(nl_w, __shfl_xor_sync(0xffffffffu, nl_w, o));
+                    for (int y = 0; y + 1 < J - x; ++y)
+                        if (ln[y + 1] < ln[y]) {
+                            const uint32_t tl = ln[y];
+                            const uint32_t* tb = lb[y];
+                            ln[y] = ln[y + 1]; lb[y] = lb[y + 1];
+                            ln[y + 1] = tl; lb[y + 1] = tb;
+                        }
+            }
+            const int nl = has ? nl_s : 0;
+            const int nl_w = nl_s;      // warp-uniform: every lane reaches the ballots below
             // chunk loop, uniform across the warp
-            uint32_t nit = (uint32_t)((hi - lo + G - 1) / G);
+            const uint32_t nit = (uint32_t)((hi - lo + G - 1) / G);
             uint32_t nit_max = nit;
+            if (VPW > 1) {
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
+                for (int o = 16; o >= G; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
+            }
             for (uint32_t it = 0; it < nit_max; ++it) {
                 const uint64_t i = lo + (uint64_t)it * G + vl;
                 const bool act = it < nit && i < hi;
@@ -336,7 +394,10 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
 #pragma unroll
                 for (int x = 0; x < J; ++x) {                                 // c-intersection (Alg. 2)
                     if (x < nl_w) {
-                        const bool pend = inter && x < nl;
+                        const bool isbm = (ln[x] & kBmFlag) != 0;
+                        if (inter && x < nl && isbm)      // hub: one bitmap load
+                            inter = (__ldg(lb[x] + (c >> 5)) >> (c & 31)) & 1u;
+                        const bool pend = inter && x < nl && !isbm;
                         const unsigned pw = __ballot_sync(0xffffffffu, pend);
                         if (pw) {
                             uint32_t pos = 0;
@@ -356,7 +417,7 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                             const unsigned pv = (pw >> vb) & kGMask;
                             const int hl = pv ? vb + 31 - __clz(pv) : lane;
                             const uint32_t mpos = __shfl_sync(0xffffffffu, pos, hl);
-                            if (pv && x < nl) { lb[x] += mpos; ln[x] -= mpos; }
+                            if (pv && x < nl && !isbm) { lb[x] += mpos; ln[x] -= mpos; }
                         }
                     }
                 }

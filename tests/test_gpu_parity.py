@@ -187,9 +187,11 @@ def test_root_range_and_slices(ctx):
     total = ctx.count("hybrid")
     assert total == oracle.count(g, q)
     l1 = ctx.stats()["level1_canonical"]
+    assert ctx.level1_size() == (l1, l1) == (oracle.level1_size(g, max(q.degrees())),) * 2
     cuts_ = [0, 7, 40, 41, l1 // 2, l1]
     for a, b in zip(cuts_, cuts_[1:]):
         ctx.set_root_range(a, b)
+        assert ctx.level1_size() == (l1, b - a)
         assert ctx.count("hybrid") == oracle.count(g, q, root_begin=a, root_end=b)
     ctx.set_root_range()
     for nparts in (2, 3, 8):
@@ -281,3 +283,26 @@ def test_alg_bytes_instrumentation(ctx):
     assert c == oracle.count(g, DENSE5[0])
     assert st["alg_bytes_extend"] > 0 and st["alg_bytes_plan"] > 0
     assert st["ms_extend"] > 0 and st["extend_launches"] >= 1
+
+
+@pytest.mark.parametrize("t", [2, 16, None])
+def test_hub_bitmaps_parity(cuts, t):
+    """SV-style hub rows (cuts_set_hub_threshold) never change a result."""
+    c = cuts(device=0, arena_bytes=1 << 30)
+    c.set_hub_threshold(t)
+    g = rmat_graph(9, 4, seed=3)
+    c.load_csr(g)
+    for q in DENSE5[::2] + SPARSE5[::3] + [named_query("C4")]:
+        want, lv = oracle.count(g, q, levels=True)
+        _set(c, q)
+        assert c.count("hybrid") == want, (t, q.name)
+        st = c.stats()
+        assert st["level_size"] == lv
+        if t is not None:
+            assert st["hubs"] == int((g.degrees() >= t).sum())
+        else:
+            assert st["hubs"] == 0
+    g = er_graph(120, 900, 3)
+    c.load_csr(g)
+    for q in DENSE5[::3]:
+        _check_full(c, g, q, modes=("hybrid",))

@@ -29,13 +29,13 @@ def run(rep):
     d = subprocess.run(['ncu', '-i', rep, '--page', 'raw', '--csv'], capture_output=True, text=True).stdout
     r = csv.reader(io.StringIO(d))
     hdr = next(r)
-    next(r)
+    units = dict(zip(hdr, next(r)))
     stalls = {}
     for row in r:
         x = dict(zip(hdr, row))
         for k in hdr:
             if k in RAW:
-                out.append(f"{k} = {x[k]}")
+                out.append(f"{k} = {x[k]} {units.get(k, '')}")
             if k.startswith('smsp__pcsamp_warps_issue_stalled_') and not k.endswith('not_issued'):
                 try:
                     v = float(x[k])
