@@ -36,7 +36,7 @@ extern "C" {
 #endif
 
 #define CUTS_MAX_K 8
-#define CUTS_ABI_VERSION 1
+#define CUTS_ABI_VERSION 2
 
 typedef struct cuts_ctx cuts_ctx;
 
@@ -88,6 +88,8 @@ typedef struct {
     uint64_t alg_bytes_plan;           /* algorithmic bytes of the plan kernels (ditto)     */
     uint64_t hubs;                     /* vertices with an adjacency bitmap (see below)     */
     uint64_t hub_threshold;            /* degree threshold used for the bitmaps             */
+    uint64_t donations;                /* work donations made (cuts_set_donation)           */
+    uint64_t donated_entries;          /* prefixes given away by those donations            */
 } cuts_stats;
 
 /* debug / instrumentation flags for cuts_set_debug */
@@ -169,6 +171,37 @@ cuts_status cuts_get_stats(const cuts_ctx* ctx, cuts_stats* out);
 
 /* Instrumentation flags (CUTS_DEBUG_*); 0 for the timed product path. */
 cuts_status cuts_set_debug(cuts_ctx* ctx, uint32_t flags);
+
+/* Seed the search with flat prefixes instead of level 1 (the receiving side of
+ * the dynamic redistribution of Alg. 3, P:1110-1144 l.16-20, "adjust depth",
+ * reading P24): d_prefixes is a DEVICE array of count rows of depth u32, row
+ * i = (f(S[0]), ..., f(S[depth-1])) in MATCHING-ORDER positions (the order in
+ * cuts_stats.order), each a partial embedding of Q[S[0..depth-1]] that passes
+ * the degree filter — e.g. rows shipped by a donor's cuts_ship_fn for the same
+ * graph and query.  Borrowed until the next count/enumerate returns.  The next
+ * count/enumerate extends exactly these prefixes (root range and slice are
+ * ignored).  1 <= depth < k, else CUTS_EINVAL; depth == 0 restores level-1
+ * seeding.  Reset by cuts_set_query.  Rows that are not valid partial
+ * embeddings give an unspecified count. */
+cuts_status cuts_set_prefixes(cuts_ctx* ctx, uint32_t depth, uint64_t count,
+                              const uint32_t* d_prefixes);
+
+/* Donation hooks (the sending side of Alg. 3).  In CUTS_HYBRID
+ * runs the library calls poll(user, depth, remaining) at every chunk boundary,
+ * where depth is the shallowest level of the DFS stack with at least two
+ * entries not yet started and remaining their number; poll returns how many of them to give
+ * away (0: none; clamped to remaining).  The library then exports the LAST
+ * `give` of those entries as flat prefixes (rows of depth u32, matching-order
+ * positions, format of cuts_set_prefixes) into arena scratch, synchronises its
+ * stream and calls ship(user, depth, d_prefixes, give); the buffer is valid
+ * only during the call (copy it out); if the arena has no room for the rows,
+ * ship is called with d_prefixes = NULL and count = 0 instead.  A non-zero return from ship aborts the
+ * count with CUTS_ECOMM.  The donated entries are never extended here, so the
+ * local count excludes them.  Both NULL (default): no donation.  Callbacks run
+ * on the calling thread. */
+typedef uint64_t (*cuts_poll_fn)(void* user, uint32_t depth, uint64_t remaining);
+typedef int (*cuts_ship_fn)(void* user, uint32_t depth, const uint32_t* d_prefixes, uint64_t count);
+cuts_status cuts_set_donation(cuts_ctx* ctx, cuts_poll_fn poll, cuts_ship_fn ship, void* user);
 
 /* Decode a trie (Fig. 3C) held in DEVICE memory: level l (0-based,
  * l < nlevels <= 8) has sizes[l] entries, candidate ids d_ca[l][x] and parent

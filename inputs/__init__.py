@@ -6,7 +6,7 @@ ordering, no intersection, no filtering, no counting), so both sides of every
 parity test can take their inputs from here without sharing method code
 (task rule ③).  The recipes are stated in DESIGN.md §3.
 """
-from .graphs import (CSRGraph, canonical_csr, er_graph, rmat_graph, cycle_graph,
+from .graphs import (CSRGraph, canonical_csr, er_graph, rmat_graph, rmat_graph_torch, cycle_graph,
                      complete_graph, path_graph, star_graph, grid_graph,
                      petersen_graph, hypercube_graph, complete_bipartite_graph,
                      graph_from_edges)
@@ -14,7 +14,7 @@ from .queries import (Query, query_from_edges, k_minus, DENSE5, SPARSE5, m11,
                       dense_family, named_query)
 
 __all__ = [
-    "CSRGraph", "canonical_csr", "er_graph", "rmat_graph", "cycle_graph",
+    "CSRGraph", "canonical_csr", "er_graph", "rmat_graph", "rmat_graph_torch", "cycle_graph",
     "complete_graph", "path_graph", "star_graph", "grid_graph", "petersen_graph",
     "hypercube_graph", "complete_bipartite_graph", "graph_from_edges",
     "Query", "query_from_edges", "k_minus", "DENSE5", "SPARSE5", "m11",

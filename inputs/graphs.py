@@ -198,3 +198,65 @@ def hypercube_graph(d: int) -> CSRGraph:
     n = 1 << d
     return graph_from_edges(n, [(v, v ^ (1 << b)) for v in range(n) for b in range(d) if v < v ^ (1 << b)],
                             name=f"Q{d}")
+
+
+# ----------------------------------------------- R-MAT, torch (same bytes, faster)
+def _i64(x: int) -> int:
+    """uint64 constant as the int64 with the same bit pattern."""
+    return x - (1 << 64) if x >= 1 << 63 else x
+
+
+def _srl(x, s: int):
+    """Logical right shift of int64 tensors viewed as uint64."""
+    import torch
+    return (x >> s) & torch.tensor((1 << (64 - s)) - 1, dtype=torch.int64, device=x.device)
+
+
+def _splitmix64_t(x):
+    z = x + _i64(0x9E3779B97F4A7C15)
+    z = (z ^ _srl(z, 30)) * _i64(0xBF58476D1CE4E5B9)
+    z = (z ^ _srl(z, 27)) * _i64(0x94D049BB133111EB)
+    return z ^ _srl(z, 31)
+
+
+def rmat_graph_torch(scale: int, ef: int, a: float = 0.57, b: float = 0.19, c: float = 0.19,
+                     seed: int = 1, device: str = "cpu", block: int = 1 << 24) -> CSRGraph:
+    """``rmat_graph`` computed with torch int64 ops (wrapping, logical shifts) —
+    byte-identical output (tests/test_oracle.py checks it), but fast enough on a
+    GPU for the scale-20/22 configs.  The relabelling permutation is numpy's."""
+    import torch
+    n = 1 << scale
+    nsamp = ef << scale
+    t1, t2, t3 = a, a + b, a + b + c
+    key = int(splitmix64(np.array([seed], dtype=np.uint64))[0])
+    key_t = torch.tensor(_i64(key), dtype=torch.int64, device=device)
+    perm_np = np.random.Generator(np.random.PCG64(seed ^ 0xA5A5)).permutation(n).astype(np.int64)
+    perm = torch.from_numpy(perm_np).to(device)
+    inv = 1.0 / float(1 << 53)
+    keys = []
+    for s0 in range(0, nsamp, block):
+        s1 = min(nsamp, s0 + block)
+        base = torch.arange(s0, s1, dtype=torch.int64, device=device) * scale
+        su = torch.zeros(s1 - s0, dtype=torch.int64, device=device)
+        du = torch.zeros_like(su)
+        for bit in range(scale):
+            r = _splitmix64_t(key_t ^ (base + bit))
+            u = _srl(r, 11).to(torch.float64) * inv
+            sbit = (u >= t2).to(torch.int64)
+            dbit = (((u >= t1) & (u < t2)) | (u >= t3)).to(torch.int64)
+            su = (su << 1) | sbit
+            du = (du << 1) | dbit
+        src, dst = perm[su], perm[du]
+        keep = src != dst
+        src, dst = src[keep], dst[keep]
+        keys.append((src << 32) | dst)
+        keys.append((dst << 32) | src)
+    k = torch.unique(torch.cat(keys)) if keys else torch.zeros(0, dtype=torch.int64, device=device)
+    rows = k >> 32
+    col = (k & 0xFFFFFFFF).to(torch.int64)
+    counts = torch.bincount(rows, minlength=n)
+    row_ptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    torch.cumsum(counts, 0, out=row_ptr[1:])
+    return CSRGraph(n=n, row_ptr=row_ptr.cpu().numpy().astype(np.uint64),
+                    col=col.cpu().numpy().astype(np.uint32),
+                    name=f"rmat_s{scale}_ef{ef}_a{a}_b{b}_c{c}_seed{seed}")

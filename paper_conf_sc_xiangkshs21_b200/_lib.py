@@ -23,7 +23,12 @@ MAX_K = 8
 # the symbols include/cuts.h declares (tests check the library exports all of them)
 EXPORTED = ["cuts_version", "cuts_create", "cuts_destroy", "cuts_last_error", "cuts_load_graph",
             "cuts_set_query", "cuts_set_root_range", "cuts_set_root_slice", "cuts_level1_size", "cuts_count",
-            "cuts_enumerate", "cuts_get_stats", "cuts_set_debug", "cuts_trie_decode", "cuts_set_hub_threshold"]
+            "cuts_enumerate", "cuts_get_stats", "cuts_set_debug", "cuts_trie_decode", "cuts_set_hub_threshold",
+            "cuts_set_prefixes", "cuts_set_donation"]
+
+# callback types of cuts_set_donation
+POLL_FN = ctypes.CFUNCTYPE(ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64)
+SHIP_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_uint64)
 
 
 class cuts_opts(ctypes.Structure):
@@ -41,7 +46,8 @@ class cuts_stats(ctypes.Structure):
                 ("ms_total", ctypes.c_double), ("ms_extend", ctypes.c_double), ("ms_plan", ctypes.c_double),
                 ("extend_launches", ctypes.c_uint64), ("alg_bytes_extend", ctypes.c_uint64),
                 ("alg_bytes_plan", ctypes.c_uint64), ("hubs", ctypes.c_uint64),
-                ("hub_threshold", ctypes.c_uint64)]
+                ("hub_threshold", ctypes.c_uint64), ("donations", ctypes.c_uint64),
+                ("donated_entries", ctypes.c_uint64)]
 
 
 _lib = None
@@ -73,6 +79,8 @@ def load() -> ctypes.CDLL:
         "cuts_set_debug": ([P, u32], i32),
         "cuts_set_hub_threshold": ([P, u32], i32),
         "cuts_trie_decode": ([P, u32, u64p, ctypes.POINTER(P), ctypes.POINTER(P), P], i32),
+        "cuts_set_prefixes": ([P, u32, u64, P], i32),
+        "cuts_set_donation": ([P, POLL_FN, SHIP_FN, P], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

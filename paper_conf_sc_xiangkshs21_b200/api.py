@@ -41,6 +41,14 @@ def default_arena_bytes(device: int, reserve: int = 4 << 30, fraction: float = 0
     return max(1 << 20, int(min(free - reserve, free * fraction)) & ~0xFFFF)
 
 
+class _DevRows:
+    """A borrowed (count, depth) int32 device buffer exposed to torch without a copy."""
+
+    def __init__(self, ptr: int, count: int, depth: int):
+        self.__cuda_array_interface__ = {"shape": (count, depth), "typestr": "<i4", "data": (ptr, False),
+                                         "version": 3, "strides": None, "stream": None}
+
+
 class Cuts:
     """One context on one device: C-ABI handle + torch-owned arena."""
 
@@ -143,6 +151,57 @@ class Cuts:
         self._check(self.lib.cuts_set_hub_threshold(self.h, 0xFFFFFFFF if t is None else int(t)))
         return self
 
+    def set_prefixes(self, rows: torch.Tensor | None):
+        """Seed the next count/enumerate with flat prefixes: rows (count, depth)
+        int32/uint32 device tensor in matching-order positions (None: level 1)."""
+        if rows is None:
+            self._prefixes = None
+            self._check(self.lib.cuts_set_prefixes(self.h, 0, 0, None))
+            return self
+        assert rows.dim() == 2 and rows.element_size() == 4 and rows.is_cuda
+        rows = rows.contiguous()
+        self._prefixes = rows                   # borrowed by the library until the next run
+        cnt, depth = rows.shape
+        self._check(self.lib.cuts_set_prefixes(self.h, depth, cnt, rows.data_ptr() if cnt else None))
+        return self
+
+    def set_donation(self, poll=None, ship=None):
+        """Donation hooks (cuts_set_donation).  poll(depth, remaining) -> int entries
+        to give; ship(depth, rows) receives a (give, depth) int32 device tensor that
+        is a COPY (owned by the callee).  None, None: off."""
+        if poll is None and ship is None:
+            self._cb = None
+            self._check(self.lib.cuts_set_donation(self.h, L.POLL_FN(), L.SHIP_FN(), None))
+            return self
+        dev = self.device
+
+        def _poll(_user, depth, remaining):
+            try:
+                return int(poll(int(depth), int(remaining)))
+            except Exception:   # never unwind through C
+                import traceback
+                traceback.print_exc()
+                return 0
+
+        def _ship(_user, depth, ptr, count):
+            try:
+                # the library synchronised its stream before the call: copy the
+                # borrowed arena rows out (zero-copy view via the CUDA array interface)
+                if not count:
+                    ship(int(depth), None)
+                    return 0
+                view = torch.as_tensor(_DevRows(ptr, int(count), int(depth)), device=dev)
+                ship(int(depth), view.clone())
+                return 0
+            except Exception:
+                import traceback
+                traceback.print_exc()
+                return 1
+
+        self._cb = (L.POLL_FN(_poll), L.SHIP_FN(_ship))
+        self._check(self.lib.cuts_set_donation(self.h, self._cb[0], self._cb[1], None))
+        return self
+
     def level1_size(self):
         """(canonical level-1 size, size inside the root range) for the current query."""
         a, b = ctypes.c_uint64(), ctypes.c_uint64()
@@ -189,6 +248,7 @@ class Cuts:
             "ms_total": s.ms_total, "ms_extend": s.ms_extend, "ms_plan": s.ms_plan,
             "extend_launches": s.extend_launches, "alg_bytes_extend": s.alg_bytes_extend,
             "alg_bytes_plan": s.alg_bytes_plan, "hubs": s.hubs, "hub_threshold": s.hub_threshold,
+            "donations": s.donations, "donated_entries": s.donated_entries,
         }
 
     def trie_decode(self, ca_levels, pa_levels) -> torch.Tensor:

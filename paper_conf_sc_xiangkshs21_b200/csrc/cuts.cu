@@ -74,6 +74,17 @@ struct cuts_ctx {
     std::vector<cudaEvent_t> ev_pool;
     size_t ev_used = 0;
     std::vector<std::pair<int, int>> ev_ext, ev_plan;
+    // flat-prefix seeding (cuts_set_prefixes): run from level pre_j instead of level 1
+    uint32_t pre_j = 0;
+    uint64_t pre_count = 0;
+    const uint32_t* pre_rows = nullptr;
+    // work donation (cuts_set_donation): DFS cursor per depth of the HYBRID stack
+    cuts_poll_fn poll = nullptr;
+    cuts_ship_fn ship = nullptr;
+    void* user = nullptr;
+    uint64_t dfs_next[kMaxK + 1] = {};   // first entry of level d not yet planned
+    uint64_t dfs_end[kMaxK + 1] = {};    // end of level d's entries still owned here
+    bool dfs_on[kMaxK + 1] = {};
 };
 
 namespace {
@@ -370,15 +381,70 @@ uint64_t pick_window(cuts_ctx* ctx, uint64_t N) {
     return std::min<uint64_t>(w, std::max<uint64_t>(N, 1));
 }
 
+void launch_export(cuts_ctx* ctx, int J, const Trie& t, uint64_t e0, uint64_t cnt, uint32_t* rows) {
+    unsigned grid = (unsigned)std::min<uint64_t>((cnt + 255) / 256, (uint64_t)ctx->num_sms * 8);
+    switch (J) {
+        case 1: k_prefix_export<1><<<grid, 256, 0, ctx->stream>>>(t, e0, cnt, rows); break;
+        case 2: k_prefix_export<2><<<grid, 256, 0, ctx->stream>>>(t, e0, cnt, rows); break;
+        case 3: k_prefix_export<3><<<grid, 256, 0, ctx->stream>>>(t, e0, cnt, rows); break;
+        case 4: k_prefix_export<4><<<grid, 256, 0, ctx->stream>>>(t, e0, cnt, rows); break;
+        case 5: k_prefix_export<5><<<grid, 256, 0, ctx->stream>>>(t, e0, cnt, rows); break;
+        case 6: k_prefix_export<6><<<grid, 256, 0, ctx->stream>>>(t, e0, cnt, rows); break;
+        case 7: k_prefix_export<7><<<grid, 256, 0, ctx->stream>>>(t, e0, cnt, rows); break;
+    }
+}
+
+// Dynamic redistribution (Alg. 3): at a chunk
+// boundary ask the caller whether an idle peer wants work; if so give away the
+// tail of the shallowest level that still has unplanned entries, exported as
+// flat prefixes (reading P24), and shrink this context's range of that level.
+cuts_status maybe_donate(cuts_ctx* ctx, Run& r) {
+    if (!ctx->poll) return CUTS_OK;
+    int d = 0;
+    for (int j = 1; j < (int)ctx->q.k; ++j)
+        if (ctx->dfs_on[j] && ctx->dfs_end[j] >= ctx->dfs_next[j] + 2) { d = j; break; }   // keep >= 1
+    if (!d) return CUTS_OK;
+    const uint64_t rem = ctx->dfs_end[d] - ctx->dfs_next[d];
+    uint64_t give = std::min<uint64_t>(ctx->poll(ctx->user, (uint32_t)d, rem), rem);
+    if (give == 0) return CUTS_OK;
+    give = std::min<uint64_t>(give, free_bytes(ctx) / 2 / (4ull * d));
+    if (give == 0) {   // no room to export: tell the caller (it may have claimed a receiver)
+        if (ctx->ship(ctx->user, (uint32_t)d, nullptr, 0) != 0) return fail(ctx, CUTS_ECOMM, "donation ship callback failed");
+        return CUTS_OK;
+    }
+    const uint64_t top_save = ctx->top;
+    uint64_t off;
+    TRY(alloc_top(ctx, give * 4ull * d, &off));
+    uint32_t* rows = (uint32_t*)(ctx->arena + off);
+    launch_export(ctx, d, r.t, ctx->dfs_end[d] - give, give, rows);
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->st.launches++;
+    const int rc = ctx->ship(ctx->user, (uint32_t)d, rows, give);
+    ctx->top = top_save;
+    if (rc != 0) return fail(ctx, CUTS_ECOMM, "donation ship callback failed (%d)", rc);
+    ctx->dfs_end[d] -= give;
+    ctx->st.donated_entries += give;
+    ctx->st.donations++;
+    return CUTS_OK;
+}
+
 // HYBRID: process entries [0, N) of level J stored at r.t.lv[J] (DFS over chunks)
 cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     const int k = (int)ctx->q.k;
     const bool last = (J == k - 1);
     const uint64_t top_save = ctx->top;
-    for (uint64_t w0 = 0; w0 < N;) {
+    ctx->dfs_on[J] = true;
+    ctx->dfs_next[J] = 0;
+    ctx->dfs_end[J] = N;
+    for (uint64_t w0 = 0;;) {
+        TRY(maybe_donate(ctx, r));
+        N = ctx->dfs_end[J];          // a donation may have shrunk this level's range
+        if (w0 >= N) break;
         Window w{};
         w.w0 = w0;
         w.W = (uint32_t)std::min<uint64_t>(pick_window(ctx, N), N - w0);
+        ctx->dfs_next[J] = w0 + w.W;
         TRY(alloc_window(ctx, J, w.W, &w));
         TRY(plan_window(ctx, r, J, w));
         if (last) {
@@ -416,19 +482,21 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
                 }
                 ctx->bot = bot_save;
                 t = t1;
+                if (t < w.total) TRY(maybe_donate(ctx, r));
             }
         }
         ctx->top = top_save;
         w0 += w.W;
     }
+    ctx->dfs_on[J] = false;
     return CUTS_OK;
 }
 
 // BFS: every level stored whole (Alg. 1); ENOMEM when a level does not fit
-cuts_status bfs_levels(cuts_ctx* ctx, Run& r, uint64_t N1) {
+cuts_status bfs_levels(cuts_ctx* ctx, Run& r, int J0, uint64_t N1) {
     const int k = (int)ctx->q.k;
     uint64_t N = N1;
-    for (int J = 1; J <= k - 1 && N > 0; ++J) {
+    for (int J = J0; J <= k - 1 && N > 0; ++J) {
         const bool last = (J == k - 1);
         const uint64_t top_save = ctx->top;
         uint64_t W = pick_window(ctx, N);
@@ -574,6 +642,25 @@ cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
     return CUTS_OK;
 }
 
+// flat-prefix seeding: levels 1..pre_j as a chain trie over the caller's rows
+cuts_status build_prefix_levels(cuts_ctx* ctx, Run& r) {
+    const uint32_t J = ctx->pre_j;
+    const uint64_t cnt = ctx->pre_count;
+    for (uint32_t l = 1; l <= J; ++l) {
+        uint64_t off;
+        TRY(alloc_bot(ctx, std::max<uint64_t>(cnt, 1) * sizeof(uint2), &off));
+        r.t.lv[l] = (uint2*)(ctx->arena + off);
+        ctx->st.level_size[l] = cnt;
+    }
+    if (cnt) {
+        unsigned grid = (unsigned)std::min<uint64_t>((cnt + 255) / 256, (uint64_t)ctx->num_sms * 8);
+        k_prefix_import<<<grid, 256, 0, ctx->stream>>>(ctx->pre_rows, J, cnt, r.t);
+        CK(cudaGetLastError());
+        ctx->st.launches++;
+    }
+    return CUTS_OK;
+}
+
 cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* rows, uint64_t cap_rows) {
     if (!ctx) return CUTS_EINVAL;
     if (!ctx->has_graph || !ctx->has_query) return fail(ctx, CUTS_ESTATE, "load_graph and set_query must precede count/enumerate");
@@ -599,9 +686,19 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     r.cap_rows = cap_rows;
     r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words};
     uint64_t n1 = 0;
+    const int k = (int)ctx->q.k;
+    for (int j = 0; j <= kMaxK; ++j) { ctx->dfs_on[j] = false; ctx->dfs_next[j] = ctx->dfs_end[j] = 0; }
+    if (ctx->pre_j) {
+        TRY(build_prefix_levels(ctx, r));
+        const int J0 = (int)ctx->pre_j;
+        if (ctx->pre_count > 0) {
+            if (mode == CUTS_BFS) TRY(bfs_levels(ctx, r, J0, ctx->pre_count));
+            else TRY(hybrid_level(ctx, r, J0, ctx->pre_count));
+        }
+        TRY(read_ctrl(ctx));
+    } else {
     TRY(build_level1(ctx, r, &n1));
     ctx->st.level_size[1] = n1;
-    const int k = (int)ctx->q.k;
     if (k == 1) {
         if (enumerate && n1 && cap_rows) {
             unsigned grid = (unsigned)std::min<uint64_t>((n1 + 255) / 256, (uint64_t)ctx->num_sms * 8);
@@ -613,11 +710,12 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
         ctx->h_ctrl[kEnumCursor] = n1;
         CK(cudaStreamSynchronize(ctx->stream));
     } else if (n1 > 0) {
-        if (mode == CUTS_BFS) TRY(bfs_levels(ctx, r, n1));
+        if (mode == CUTS_BFS) TRY(bfs_levels(ctx, r, 1, n1));
         else TRY(hybrid_level(ctx, r, 1, n1));
         TRY(read_ctrl(ctx));
     } else {
         TRY(read_ctrl(ctx));
+    }
     }
     if (enumerate) {
         ctx->st.count_lo = ctx->h_ctrl[kEnumCursor];
@@ -756,7 +854,39 @@ cuts_status cuts_set_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr, c
     ctx->slice_end = ~0ull;
     ctx->part = 0;
     ctx->nparts = 1;
+    ctx->pre_j = 0;
+    ctx->pre_count = 0;
+    ctx->pre_rows = nullptr;
     ctx->has_query = true;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_prefixes(cuts_ctx* ctx, uint32_t depth, uint64_t count, const uint32_t* d_prefixes) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (!ctx->has_query) return fail(ctx, CUTS_ESTATE, "cuts_set_query must precede cuts_set_prefixes");
+    if (depth == 0) {                    // back to level-1 seeding
+        ctx->pre_j = 0;
+        ctx->pre_count = 0;
+        ctx->pre_rows = nullptr;
+        return CUTS_OK;
+    }
+    if (depth >= ctx->q.k) return fail(ctx, CUTS_EINVAL, "prefix depth %u must be < k = %u", depth, ctx->q.k);
+    if (count && !d_prefixes) return fail(ctx, CUTS_EINVAL, "null prefix rows");
+    if (count > kMaxLevel) return fail(ctx, CUTS_EINVAL, "too many prefixes (%llu)", (unsigned long long)count);
+    ctx->pre_j = depth;
+    ctx->pre_count = count;
+    ctx->pre_rows = d_prefixes;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_donation(cuts_ctx* ctx, cuts_poll_fn poll, cuts_ship_fn ship, void* user) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if ((poll == nullptr) != (ship == nullptr)) return fail(ctx, CUTS_EINVAL, "poll and ship must both be set or both NULL");
+    ctx->poll = poll;
+    ctx->ship = ship;
+    ctx->user = user;
     return CUTS_OK;
 }
 

@@ -360,7 +360,7 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                     }
                 }
             }
-            if (nl_s > 1) {
+            if (nl_s > 0) {   // also for one list: moves it into slot 0 (the loop below reads slots < nl_s)
 #pragma unroll
                 for (int x = 0; x < J; ++x)
 #pragma unroll
@@ -455,6 +455,38 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
         if (lane == 0) atomicAdd(ctrl + kBytesExt, bytes);
     }
     (void)vb;
+}
+
+// ---------------------------------------------------------- work donation
+// Flat prefixes (reading P24): a donated unit of work is a J-vertex partial
+// embedding in matching-order positions, rows of J u32.  Export walks the trie
+// of the donor (the path recovery of P:956-958); import rebuilds a chain trie
+// (level l entry i = (row[i][l-1], parent i)) that the receiver extends from
+// level J on, so no trie is shipped (cf. the extraction cost named at P:1168-1176).
+template <int J>
+__global__ void k_prefix_export(Trie t, uint64_t e0, uint64_t cnt, uint32_t* __restrict__ rows) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        uint2 cur = t.lv[J][e0 + i];
+        uint32_t* row = rows + i * J;
+        row[J - 1] = cur.x;
+        uint32_t idx = cur.y;
+#pragma unroll
+        for (int p = J - 2; p >= 0; --p) {
+            cur = t.lv[p + 1][idx];
+            row[p] = cur.x;
+            idx = cur.y;
+        }
+    }
+}
+
+// lv[l] (l = 1..J) each hold cnt entries: (rows[i][l-1], i)
+__global__ void k_prefix_import(const uint32_t* __restrict__ rows, uint32_t J, uint64_t cnt, Trie t) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        for (uint32_t l = 1; l <= J; ++l)
+            const_cast<uint2*>(t.lv[l])[i] = make_uint2(rows[i * J + l - 1], (uint32_t)i);
+    }
 }
 
 // ---------------------------------------------------------------- trie decode

@@ -43,7 +43,7 @@ def test_library_exports_every_declared_symbol(lib):
 
 def test_version_and_null_args(lib):
     lib.cuts_version.restype = ctypes.c_int
-    assert lib.cuts_version() == 1
+    assert lib.cuts_version() == 2
     lib.cuts_create.restype = ctypes.c_int
     lib.cuts_create.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
     assert lib.cuts_create(None, None) == -1                  # CUTS_EINVAL, no CUDA call

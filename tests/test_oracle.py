@@ -299,3 +299,12 @@ def test_fig3_trie_decode_matches_csf():
         walk(0, x, ())
     assert got == paths
     assert len(got) == 8 and got[0] == (0, 3, 2, 5) and got[-1] == (1, 2, 3, 4)
+
+
+def test_rmat_torch_generator_is_byte_identical():
+    """The torch R-MAT generator (used for the scale-20/22 configs) must emit the
+    same canonical CSR bytes as the numpy reference generator."""
+    from inputs import rmat_graph_torch
+    for args in [(10, 8, 0.57, 0.19, 0.19, 3), (11, 16, 0.45, 0.22, 0.22, 1), (9, 4, 0.35, 0.22, 0.22, 7)]:
+        a, b = rmat_graph(*args), rmat_graph_torch(*args, block=1 << 12)
+        assert np.array_equal(a.row_ptr, b.row_ptr) and np.array_equal(a.col, b.col), args

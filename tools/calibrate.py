@@ -18,7 +18,7 @@ sys.path.insert(0, ROOT)
 
 import torch  # noqa: E402
 
-from inputs import rmat_graph, DENSE5, SPARSE5, dense_family  # noqa: E402
+from inputs import rmat_graph_torch, DENSE5, SPARSE5, dense_family  # noqa: E402
 from paper_conf_sc_xiangkshs21_b200 import Cuts  # noqa: E402
 
 
@@ -32,6 +32,8 @@ def main():
     ap.add_argument("--budget", type=float, default=20.0, help="seconds allowed for a full run")
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--out", default="")
+    ap.add_argument("--min-nparts", type=int, default=1)
+    ap.add_argument("--max-nparts", type=int, default=4096)
     args = ap.parse_args()
     if args.family == "c2":
         queries = DENSE5 + SPARSE5
@@ -41,11 +43,12 @@ def main():
     for abc in args.abc or ["0.57,0.19,0.19"]:
         a, b, c = map(float, abc.split(","))
         t = time.time()
-        g = rmat_graph(args.scale, args.ef, a, b, c, seed=args.seed)
+        g = rmat_graph_torch(args.scale, args.ef, a, b, c, seed=args.seed, device="cuda")
         gen_s = time.time() - t
         d = g.degrees()
         ctx.load_csr(g)
-        line = json.dumps({"graph": g.name, "n": g.n, "m": g.m, "maxdeg": int(d.max()), "gen_s": round(gen_s, 1)})
+        line = json.dumps({"graph": g.name, "n": g.n, "m": g.m, "maxdeg": int(d.max()), "gen_s": round(gen_s, 1),
+                           "isolated": int((d == 0).sum()), "deg_ge7": int((d >= 7).sum())})
         print(line, flush=True)
         if args.out:
             with open(args.out, "a") as f:
@@ -54,7 +57,7 @@ def main():
             qr, qc = q.csr()
             ctx.set_query(qr, qc)
             rec = {"q": q.name}
-            for nparts in (4096, 512, 64, 8, 1):
+            for nparts in [p for p in (32768, 4096, 512, 64, 8, 1) if args.min_nparts <= p <= args.max_nparts]:
                 ctx.set_root_slice(0, 2**64 - 1, 0, nparts)
                 torch.cuda.synchronize()
                 t = time.time()
