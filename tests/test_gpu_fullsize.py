@@ -1,0 +1,86 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py times.
+
+The bench runs every query of a workload through ``Cuts(device, stream)`` with
+the default arena (most of the free HBM) in HYBRID mode.  Full counts at these
+sizes are out of the oracle's reach, so the outputs are sampled (SURVEY §8.d,
+"parity plan"):
+
+* root ranges: the exact count over a few short ranges of the canonical
+  level-1 list (evenly spaced, plus the range holding the max-degree root when
+  the query is cheap there) — GPU and oracle on the same range, bit-exact;
+* closed forms that hold at any size: stars K_{1,s} and paths P3 depend only on
+  the degree sequence (sum_v d(d-1)...(d-s+1)), so the full-scale GPU count is
+  checked against exact integer arithmetic on the graph's degrees.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from inputs import named_query
+from workloads import WORKLOADS
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def bench_ctx():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_xiangkshs21_b200 import Cuts
+    stream = torch.cuda.Stream(device=0)
+    return Cuts(device=0, stream=stream)      # bench.py's configuration: default arena, own stream
+
+
+def _set(ctx, q):
+    qr, qc = q.csr()
+    ctx.set_query(qr, qc)
+
+
+def _falling(d, s):
+    """sum_v d(v)(d(v)-1)...(d(v)-s+1) in exact Python integers."""
+    tot = 0
+    for x in d.tolist():
+        p = 1
+        for i in range(s):
+            p *= x - i
+        if p > 0:
+            tot += p
+    return tot
+
+
+def _ranges(l1, width, nsamples):
+    starts = np.linspace(0, max(0, l1 - width), nsamples).astype(np.int64)
+    return sorted({(int(s), int(min(l1, s + width))) for s in starts})
+
+
+@pytest.mark.parametrize("part", [0, 1])
+def test_c2_full_size_root_ranges(bench_ctx, part):
+    wl = WORKLOADS["C2"]
+    spec, qs = wl.parts[part]
+    g = spec.build()
+    bench_ctx.load_csr(g, validate=True)
+    for q in qs:
+        _set(bench_ctx, q)
+        l1, _ = bench_ctx.level1_size()
+        assert l1 == oracle.level1_size(g, max(q.degrees()))
+        for a, b in _ranges(l1, 3, 5):
+            bench_ctx.set_root_range(a, b)
+            got = bench_ctx.count(wl.mode)
+            want = oracle.count(g, q, root_begin=a, root_end=b)
+            assert got == want, (spec.name, q.name, a, b, got, want)
+        bench_ctx.set_root_range()
+
+
+@pytest.mark.parametrize("part", [0, 1])
+def test_c2_full_size_closed_forms(bench_ctx, part):
+    spec, _ = WORKLOADS["C2"].parts[part]
+    g = spec.build()
+    bench_ctx.load_csr(g)
+    d = g.degrees().astype(np.int64)
+    for name, s in (("P3", 2), ("S3", 3), ("K1_4", 4)):
+        q = named_query(name)
+        _set(bench_ctx, q)
+        want = _falling(d, s)
+        got = bench_ctx.count("hybrid")
+        assert got == want, (spec.name, name, got, want)
