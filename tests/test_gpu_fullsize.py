@@ -78,7 +78,9 @@ def test_c2_full_size_closed_forms(bench_ctx, part):
     g = spec.build()
     bench_ctx.load_csr(g)
     d = g.degrees().astype(np.int64)
-    for name, s in (("P3", 2), ("S3", 3), ("K1_4", 4)):
+    # K1_4 on the dense-family graph is ~3e13 embeddings (minutes): stars up to
+    # K1_3 there, K1_4 on the sparse-family graph (4e11, seconds)
+    for name, s in (("P3", 2), ("S3", 3)) + ((("K1_4", 4),) if part == 1 else ()):
         q = named_query(name)
         _set(bench_ctx, q)
         want = _falling(d, s)

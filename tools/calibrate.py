@@ -34,11 +34,15 @@ def main():
     ap.add_argument("--out", default="")
     ap.add_argument("--min-nparts", type=int, default=1)
     ap.add_argument("--max-nparts", type=int, default=4096)
+    ap.add_argument("--only", default="", help="comma list of query names to keep")
     args = ap.parse_args()
     if args.family == "c2":
         queries = DENSE5 + SPARSE5
     else:
         queries = [q for k in map(int, args.family.split(",")) for q in dense_family(k)]
+    if args.only:
+        keep = set(args.only.split(","))
+        queries = [q for q in queries if q.name in keep]
     ctx = Cuts(device=0)
     for abc in args.abc or ["0.57,0.19,0.19"]:
         a, b, c = map(float, abc.split(","))
