@@ -10,7 +10,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libcuts.so")
+LIB_PATH = os.environ.get("CUTS_LIB") or os.path.join(_HERE, "libcuts.so")   # CUTS_LIB: A/B builds
 
 CUTS_OK, CUTS_EINVAL, CUTS_ENOMEM, CUTS_ECUDA = 0, -1, -2, -3
 CUTS_EOVERFLOW, CUTS_ETRUNC, CUTS_ESTATE, CUTS_EUNSUPPORTED, CUTS_ECOMM = -4, -5, -6, -7, -8

@@ -225,6 +225,8 @@ struct Window {
     uint32_t W;
     uint32_t* path;
     uint64_t* src;
+    uint64_t* lst_off;   // (J-1) x W list descriptors from k_plan
+    uint32_t* lst_len;
     uint64_t* ub;
     uint64_t* offs;
     void* cub_tmp;
@@ -234,7 +236,7 @@ struct Window {
 
 template <int J>
 void launch_plan_t(cuts_ctx* ctx, const Graph& g, const Trie& t, const Window& w, int grid) {
-    k_plan<J><<<grid, 256, 0, ctx->stream>>>(g, t, ctx->q, w.w0, w.W, w.path, w.src, w.ub, ctx->ctrl,
+    k_plan<J><<<grid, 256, 0, ctx->stream>>>(g, t, ctx->q, w.w0, w.W, w.path, w.src, w.ub, w.lst_off, w.lst_len, ctx->ctrl,
                                              (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0);
 }
 
@@ -251,12 +253,12 @@ void launch_plan(cuts_ctx* ctx, int J, const Graph& g, const Trie& t, const Wind
     }
 }
 
-template <int J, int M, int G>
+template <int J, int NL, int M, int G>
 void launch_extend_g(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
     static int occ = 0;
     if (!occ) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<J, M, G>, 256, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_extend<J, NL, M, G>, 256, 0);
         if (occ < 1) occ = 1;
     }
     // persistent-style grid: every resident CTA slot, entries fetched dynamically
@@ -265,19 +267,36 @@ void launch_extend_g(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0
     // entries per virtual-warp fetch: ~2K candidate items per atomic on the work counter
     const double avg = (double)w.total / (double)std::max<uint32_t>(w.W, 1);
     const uint32_t batch = (uint32_t)std::min(256.0, std::max(2.0, 2048.0 / std::max(avg, 1.0) / (32 / G)));
-    k_extend<J, M, G><<<(unsigned)grid, 256, 0, ctx->stream>>>(g, ctx->q, w.w0, w.W, w.path, w.src, w.offs, t0, t1,
-                                                               out_level, out_rows, cap, ctx->ctrl,
-                                                               (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0, batch);
+    k_extend<J, NL, M, G><<<(unsigned)grid, 256, 0, ctx->stream>>>(g, ctx->q, w.w0, w.W, w.path, w.src, w.offs,
+                                                                   w.lst_off, w.lst_len, t0, t1,
+                                                                   out_level, out_rows, cap, ctx->ctrl,
+                                                                   (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0, batch);
 }
 
+template <int J, int NL, int M>
+void launch_extend_nl(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
+                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
+    // virtual-warp width from the average candidate-list length (P:911-916)
+    const double avg = (double)w.total / (double)std::max<uint32_t>(w.W, 1);
+    if (avg >= 96) launch_extend_g<J, NL, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else if (avg >= 24) launch_extend_g<J, NL, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else launch_extend_g<J, NL, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+}
+
+// NL = |bw[J]| - 1 lists to test besides the source: a compile-time constant per level
 template <int J, int M>
 void launch_extend_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
-    // virtual-warp width from the average candidate-list length (P:911-916)
-    const double avg = (double)w.total / (double)std::max<uint32_t>(w.W, 1);
-    if (avg >= 96) launch_extend_g<J, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
-    else if (avg >= 24) launch_extend_g<J, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
-    else launch_extend_g<J, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    const int nl = __builtin_popcount(ctx->q.bw[J]) - 1;
+    switch (nl) {
+        case 0: launch_extend_nl<J, 0, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 1: if constexpr (J > 1) launch_extend_nl<J, (J > 1 ? 1 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 2: if constexpr (J > 2) launch_extend_nl<J, (J > 2 ? 2 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 3: if constexpr (J > 3) launch_extend_nl<J, (J > 3 ? 3 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 4: if constexpr (J > 4) launch_extend_nl<J, (J > 4 ? 4 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 5: if constexpr (J > 5) launch_extend_nl<J, (J > 5 ? 5 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+        case 6: if constexpr (J > 6) launch_extend_nl<J, (J > 6 ? 6 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
+    }
 }
 
 template <int M>
@@ -306,7 +325,9 @@ struct Run {
 };
 
 uint64_t window_scratch_bytes(uint64_t W, int J, size_t cub_bytes) {
-    return align_up((uint64_t)J * W * 4) + align_up(W * 8) + 2 * align_up((W + 1) * 8) + align_up(cub_bytes) + 4 * kAlign;
+    const uint64_t nl = (uint64_t)std::max(J - 1, 1);
+    return align_up((uint64_t)J * W * 4) + align_up(W * 8) + 2 * align_up((W + 1) * 8) + align_up(nl * W * 8) +
+           align_up(nl * W * 4) + align_up(cub_bytes) + 6 * kAlign;
 }
 
 cuts_status read_ctrl(cuts_ctx* ctx) {
@@ -366,6 +387,9 @@ cuts_status alloc_window(cuts_ctx* ctx, int J, uint64_t W, Window* w) {
     w->src = (uint64_t*)p; p += align_up(W * 8);
     w->ub = (uint64_t*)p; p += align_up((W + 1) * 8);
     w->offs = (uint64_t*)p; p += align_up((W + 1) * 8);
+    const uint64_t nl = (uint64_t)std::max(J - 1, 1);
+    w->lst_off = (uint64_t*)p; p += align_up(nl * W * 8);
+    w->lst_len = (uint32_t*)p; p += align_up(nl * W * 4);
     w->cub_tmp = p;
     w->cub_bytes = cub_bytes;
     return CUTS_OK;
@@ -373,7 +397,7 @@ cuts_status alloc_window(cuts_ctx* ctx, int J, uint64_t W, Window* w) {
 
 // window size for depth J: bounded so all depths' scratch takes <= 1/8 of the arena
 uint64_t pick_window(cuts_ctx* ctx, uint64_t N) {
-    uint64_t per = (uint64_t)(ctx->q.k) * 4 + 24;   // path + src + ub + offs per entry
+    uint64_t per = (uint64_t)(ctx->q.k) * 4 + 24 + (uint64_t)std::max<int>((int)ctx->q.k - 2, 1) * 12;   // path + src + ub + offs + list descriptors
     uint64_t budget = ctx->arena_bytes / 8 / std::max<uint32_t>(1, ctx->q.k - 1);
     uint64_t w = budget / per;
     w = std::max<uint64_t>(w, 1);

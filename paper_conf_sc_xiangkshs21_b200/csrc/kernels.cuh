@@ -194,11 +194,22 @@ __global__ void k_rows_k1(const uint2* __restrict__ L1, uint64_t cnt, uint32_t* 
 
 // ---------------------------------------------------------------- plan
 // J = number of matched positions of the entries (= next position to match).
+// One thread per entry: walk the trie path, read the bounds of the
+// backward-neighbour lists bw[J], take the shortest as the candidate source
+// (c-intersection initial set, Alg. 2 l.22-23) and emit ub(e) = its length, a
+// never-exceeded bound on the entry's children.  The other lists are written
+// as descriptors sorted by length (shortest first; hub lists as bitmap rows,
+// which sort last), so the extend kernel's virtual warps read them instead of
+// recomputing them lane-redundantly.
+//   lst_off[x*W + e]: element offset into col (or into bm for a bitmap row)
+//   lst_len[x*W + e]: list length, | kBmFlag for a bitmap row
 template <int J>
 __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t w0, uint32_t W,
                                               uint32_t* __restrict__ path_s,
                                               uint64_t* __restrict__ src_off,
                                               uint64_t* __restrict__ ub,
+                                              uint64_t* __restrict__ lst_off,
+                                              uint32_t* __restrict__ lst_len,
                                               unsigned long long* __restrict__ ctrl, int count_bytes) {
     const uint32_t bw = q.bw[J];
     unsigned long long bytes_plan = 0, bytes_ext = 0;
@@ -214,20 +225,55 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
             path[p] = cur.x;
             idx = cur.y;
         }
-        uint64_t best = ~0ull, bsrc = 0, lists = 0;
+        uint64_t lb_[J];
+        uint32_t ln_[J];
+        uint64_t lists = 0, best_b = 0;
+        uint32_t best_d = 0xffffffffu;
+        int best = -1;
 #pragma unroll
         for (int p = 0; p < J; ++p) {
+            ln_[p] = 0xffffffffu;
+            lb_[p] = 0;
             if ((bw >> p) & 1u) {
-                uint64_t b = g.row_ptr[path[p]];
-                uint64_t d = g.row_ptr[path[p] + 1] - b;
+                const uint64_t b = g.row_ptr[path[p]];
+                const uint32_t d = (uint32_t)(g.row_ptr[path[p] + 1] - b);
                 lists += d;
-                if (d < best) { best = d; bsrc = b; }
+                lb_[p] = b;
+                ln_[p] = d;
+                if (best < 0 || d < best_d) { best = p; best_d = d; best_b = b; }
+            }
+        }
+        src_off[e] = best_b;
+        ub[e] = best_d;
+        // other lists: hub rows become bitmap probes; then sort by length
+        int x = 0;
+#pragma unroll
+        for (int p = 0; p < J; ++p) {
+            if (p != best && ((bw >> p) & 1u)) {
+                const uint32_t h = g.hub ? __ldg(g.hub + path[p]) : kNoHub;
+                if (h != kNoHub) { lb_[p] = (uint64_t)h * g.words; ln_[p] |= kBmFlag; }
+            } else {
+                ln_[p] = 0xffffffffu;     // not a list to test (the source, or not backward)
             }
         }
 #pragma unroll
+        for (int i = 0; i < J; ++i)
+#pragma unroll
+            for (int y = 0; y + 1 < J - i; ++y)
+                if (ln_[y + 1] < ln_[y]) {
+                    const uint32_t tl = ln_[y]; ln_[y] = ln_[y + 1]; ln_[y + 1] = tl;
+                    const uint64_t tb = lb_[y]; lb_[y] = lb_[y + 1]; lb_[y + 1] = tb;
+                }
+        const int nl = __popc(bw) - 1;
+#pragma unroll
+        for (int y = 0; y < J - 1; ++y)
+            if (y < nl) {
+                lst_off[(size_t)y * W + e] = lb_[y];
+                lst_len[(size_t)y * W + e] = ln_[y];
+            }
+        (void)x;
+#pragma unroll
         for (int p = 0; p < J; ++p) path_s[(size_t)p * W + e] = path[p];
-        src_off[e] = bsrc;
-        ub[e] = best;
         if (count_bytes) {   // 8 (entry) + 8(J-1) (hops) + 16 per list bound
             bytes_plan += 8ull + 8ull * (J - 1) + 16ull * __popc(bw);
             bytes_ext += 4ull * lists;                   // every backward list read once
@@ -244,42 +290,31 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
 }
 
 // ---------------------------------------------------------------- extend
-// lower bound of c in sorted col[b, e): first position p with col[p] >= c
-__device__ __forceinline__ uint64_t lower_bound_u32(const uint32_t* __restrict__ col, uint64_t b, uint64_t e,
-                                                    uint32_t c) {
-    uint64_t len = e - b;
-    const uint32_t* base = col + b;
-    while (len > 0) {
-        uint64_t half = len >> 1;
-        if (__ldg(base + half) < c) { base += half + 1; len -= half + 1; }
-        else len = half;
-    }
-    return (uint64_t)(base - col);
-}
-
-
 // Items [t0, t1) of the window's flat candidate space (offs = exclusive scan of
 // ub, W+1 entries, ub(e) = |source list|).  J = matched positions of the
-// parents; the child takes position J.
+// parents; the child takes position J.  NL = |bw[J]| - 1 lists to test besides
+// the source (a compile-time constant per level).
 //
 // Mapping: a virtual warp of G lanes per entry (the paper's single-bin virtual
 // warps sized from the average degree), entries fetched dynamically
-// in batches.  Per entry the path and the backward lists' bounds are loaded
-// once into registers (uniform across the virtual warp); the G lanes walk the
-// source list G candidates at a time (coalesced), apply injectivity and the
-// degree filter, then test membership in the other backward lists, shortest
-// first, each by a binary search that starts at a per-list cursor which only
-// moves forward (candidates arrive in ascending order).  Output: one ballot per
-// warp and one atomic per warp per chunk.
+// in batches.  The G lanes walk the source list G candidates at a time
+// (coalesced), apply injectivity and the degree filter (Def. 5),
+// probe the hub lists' bitmaps (loads issued together), then test membership
+// in the remaining sorted lists, shortest first, each by a branch-free binary
+// search from a per-list cursor that only moves forward (candidates arrive in
+// ascending order).  Output: one ballot and one atomic per warp per chunk
+// (P:704-708).
 //
 // M: kWrite -> level J+1 entries (vertex, parent = w0 + e) at ctrl[kCursor]
 // (dropped past cap; HYBRID sizes cap so that never happens); kCount -> 128-bit
 // count; kEnum -> rows of k u32 in query-id order at ctrl[kEnumCursor].
-template <int J, int M, int G>
+template <int J, int NL, int M, int G>
 __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
                                                const uint32_t* __restrict__ path_s,
                                                const uint64_t* __restrict__ src_off,
                                                const uint64_t* __restrict__ offs,
+                                               const uint64_t* __restrict__ lst_off,
+                                               const uint32_t* __restrict__ lst_len,
                                                uint64_t t0, uint64_t t1,
                                                uint2* __restrict__ out_level,
                                                uint32_t* __restrict__ out_rows, uint64_t cap,
@@ -287,6 +322,7 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                                                uint32_t batch) {
     constexpr int VPW = 32 / G;
     constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
+    constexpr int NLA = NL > 0 ? NL : 1;
     __shared__ uint32_t s_ent[2];
     if (threadIdx.x == 0) {        // entries holding items t0 and t1-1
         uint64_t tt[2] = {t0, t1 - 1};
@@ -305,11 +341,10 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
     const int lane = threadIdx.x & 31;
     const int vl = lane & (G - 1);
     const int vb = lane & ~(G - 1);
-    const uint32_t bw = q.bw[J];
     const uint32_t qd = q.qdeg[J];
-    const int nl_s = __popc(bw) - 1;   // lists besides the source (same for every entry)
     unsigned long long my_count = 0, bytes = 0;
     unsigned int* work = (unsigned int*)(ctrl + kWork);
+    const unsigned long long wbytes = M == kCount ? 0ull : (M == kEnum ? 4ull * q.k : 8ull);
 
     for (;;) {
         uint32_t base = 0;
@@ -323,106 +358,39 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
             const bool has = ei < nent;
             const uint32_t e = ea + (has ? ei : 0);
             // this entry's item range, clipped to [t0, t1)
-            uint64_t lo = 0, hi = 0;
+            uint32_t ilo = 0, ihi = 0;
+            uint64_t so = 0;
+            uint32_t path[J];
+            const uint32_t* lb[NLA];   // list cursors (advance)
+            uint32_t ln[NLA];          // remaining lengths (| kBmFlag: bitmap row)
             if (has) {
                 const uint64_t o0 = offs[e], o1 = offs[e + 1];
-                lo = (o0 > t0 ? o0 : t0) - o0;
-                hi = (o1 < t1 ? o1 : t1) - o0;
-            }
-            const uint64_t so = has ? src_off[e] : 0;
-            uint32_t path[J];
+                ilo = (uint32_t)((o0 > t0 ? o0 : t0) - o0);
+                ihi = (uint32_t)((o1 < t1 ? o1 : t1) - o0);
+                so = src_off[e];
 #pragma unroll
-            for (int p = 0; p < J; ++p) path[p] = has ? path_s[(size_t)p * W + e] : 0xffffffffu;
-            // other backward lists (all but the source), sorted by length ascending;
-            // fixed register slots (compile-time indices), unused slots sort last
-            const uint32_t* lb[J];     // list cursor (advances)
-            uint32_t ln[J];            // remaining length; unused slots sort last
+                for (int p = 0; p < J; ++p) path[p] = path_s[(size_t)p * W + e];
 #pragma unroll
-            for (int p = 0; p < J; ++p) {
-                lb[p] = g.col;
-                ln[p] = 0xffffffffu;
-            }
-            if (nl_s > 0 && has) {
-#pragma unroll
-                for (int p = 0; p < J; ++p) {
-                    if ((bw >> p) & 1u) {
-                        const uint64_t b = g.row_ptr[path[p]];
-                        if (b != so) {
-                            const uint32_t h = g.hub ? __ldg(g.hub + path[p]) : kNoHub;
-                            if (h != kNoHub) {     // hub list: probe its bitmap row (sorts last)
-                                lb[p] = g.bm + (uint64_t)h * g.words;
-                                ln[p] = kBmFlag | (uint32_t)(g.row_ptr[path[p] + 1] - b);
-                            } else {
-                                lb[p] = g.col + b;
-                                ln[p] = (uint32_t)(g.row_ptr[path[p] + 1] - b);
-                            }
-                        }
-                    }
+                for (int x = 0; x < NL; ++x) {
+                    const uint64_t off = lst_off[(size_t)x * W + e];
+                    ln[x] = lst_len[(size_t)x * W + e];
+                    lb[x] = ((ln[x] & kBmFlag) ? g.bm : g.col) + off;
                 }
-            }
-            if (nl_s > 0) {   // also for one list: moves it into slot 0 (the loop below reads slots < nl_s)
+            } else {
 #pragma unroll
-                for (int x = 0; x < J; ++x)
+                for (int p = 0; p < J; ++p) path[p] = 0xffffffffu;
 #pragma unroll
-                    for (int y = 0; y + 1 < J - x; ++y)
-                        if (ln[y + 1] < ln[y]) {
-                            const uint32_t tl = ln[y];
-                            const uint32_t* tb = lb[y];
-                            ln[y] = ln[y + 1]; lb[y] = lb[y + 1];
-                            ln[y + 1] = tl; lb[y + 1] = tb;
-                        }
+                for (int x = 0; x < NLA; ++x) { ln[x] = 0; lb[x] = g.col; }
             }
-            const int nl = has ? nl_s : 0;
-            const int nl_w = nl_s;      // warp-uniform: every lane reaches the ballots below
-            // chunk loop, uniform across the warp
-            const uint32_t nit = (uint32_t)((hi - lo + G - 1) / G);
+            const uint32_t* __restrict__ src = g.col + so;
+            const uint32_t nit = (ihi - ilo + G - 1) / G;
             uint32_t nit_max = nit;
             if (VPW > 1) {
 #pragma unroll
                 for (int o = 16; o >= G; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
             }
-            for (uint32_t it = 0; it < nit_max; ++it) {
-                const uint64_t i = lo + (uint64_t)it * G + vl;
-                const bool act = it < nit && i < hi;
-                const uint32_t c = act ? __ldg(g.col + so + i) : 0u;
-                bool inj = act;
-#pragma unroll
-                for (int p = 0; p < J; ++p) inj = inj && (path[p] != c);      // injectivity (P:211-216)
-                bool ok = inj && (qd <= 1 || __ldg(g.deg + c) >= qd);       // degree filter (Def. 5);
-                                                                              // every neighbour has deg >= 1
-                bool inter = count_bytes ? act : ok;
-#pragma unroll
-                for (int x = 0; x < J; ++x) {                                 // c-intersection (Alg. 2)
-                    if (x < nl_w) {
-                        const bool isbm = (ln[x] & kBmFlag) != 0;
-                        if (inter && x < nl && isbm)      // hub: one bitmap load
-                            inter = (__ldg(lb[x] + (c >> 5)) >> (c & 31)) & 1u;
-                        const bool pend = inter && x < nl && !isbm;
-                        const unsigned pw = __ballot_sync(0xffffffffu, pend);
-                        if (pw) {
-                            uint32_t pos = 0;
-                            if (pend) {     // branch-free lower bound from the cursor
-                                const uint32_t* b0 = lb[x];
-                                uint32_t len = ln[x];
-                                while (len > 1) {
-                                    const uint32_t half = len >> 1;
-                                    b0 = (__ldg(b0 + half - 1) < c) ? b0 + half : b0;
-                                    len -= half;
-                                }
-                                inter = len == 1 && __ldg(b0) == c;
-                                pos = (uint32_t)(b0 - lb[x]);
-                            }
-                            // candidates ascend with the lane, so the highest pending lane of
-                            // the virtual warp holds the furthest safe cursor position
-                            const unsigned pv = (pw >> vb) & kGMask;
-                            const int hl = pv ? vb + 31 - __clz(pv) : lane;
-                            const uint32_t mpos = __shfl_sync(0xffffffffu, pos, hl);
-                            if (pv && x < nl && !isbm) { lb[x] += mpos; ln[x] -= mpos; }
-                        }
-                    }
-                }
-                if (count_bytes) bytes += (inter ? 4ull : 0ull) + (inter && ok && M != kCount ? (M == kEnum ? 4ull * q.k : 8ull) : 0ull);
-                ok = ok && inter;
+            // output of one candidate per lane: warp-aggregated slots
+            auto emit = [&](bool ok, uint32_t c) {
                 if (M == kCount) {
                     my_count += ok ? 1 : 0;
                 } else {
@@ -443,6 +411,80 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                         }
                     }
                 }
+            };
+            if constexpr (NL == 0) {
+                // one backward list: it is the source, so the intersection is the list
+                // itself and only injectivity + degree remain; two candidates per lane per
+                // iteration, loads issued together
+#pragma unroll 1
+                for (uint32_t it = 0; it < nit_max; it += 2) {
+                    const uint32_t i0 = ilo + it * G + vl, i1 = i0 + G;
+                    const bool a0 = i0 < ihi, a1 = i1 < ihi;
+                    const uint32_t c0 = a0 ? __ldg(src + i0) : 0u;
+                    const uint32_t c1 = a1 ? __ldg(src + i1) : 0u;
+                    bool k0 = a0, k1 = a1;
+#pragma unroll
+                    for (int p = 0; p < J; ++p) { k0 = k0 && (path[p] != c0); k1 = k1 && (path[p] != c1); }
+                    if (qd > 1) {
+                        const uint32_t d0 = k0 ? __ldg(g.deg + c0) : 0u;
+                        const uint32_t d1 = k1 ? __ldg(g.deg + c1) : 0u;
+                        k0 = k0 && d0 >= qd;
+                        k1 = k1 && d1 >= qd;
+                    }
+                    if (count_bytes)
+                        bytes += (a0 ? 4ull : 0ull) + (a1 ? 4ull : 0ull) + (k0 ? wbytes : 0ull) + (k1 ? wbytes : 0ull);
+                    emit(k0, c0);
+                    if (it + 1 < nit_max) emit(k1, c1);
+                }
+            } else {
+            for (uint32_t it = 0; it < nit_max; ++it) {
+                const uint32_t i = ilo + it * G + vl;
+                const bool act = i < ihi;
+                const uint32_t c = act ? __ldg(src + i) : 0u;
+                bool inj = act;
+#pragma unroll
+                for (int p = 0; p < J; ++p) inj = inj && (path[p] != c);      // injectivity (P:211-216)
+                // independent loads issued together: degree (Def. 5) and every hub-bitmap probe
+                const bool pre = count_bytes ? act : inj;
+                const uint32_t dg = (inj && qd > 1) ? __ldg(g.deg + c) : 0xffffffffu;
+                uint32_t bmw[NLA];
+#pragma unroll
+                for (int x = 0; x < NL; ++x)
+                    bmw[x] = (pre && (ln[x] & kBmFlag)) ? __ldg(lb[x] + (c >> 5)) : 0xffffffffu;
+                bool ok = inj && dg >= qd;                                    // every neighbour has deg >= 1
+                bool inter = count_bytes ? act : ok;
+#pragma unroll
+                for (int x = 0; x < NL; ++x)                                  // c-intersection (Alg. 2): hubs
+                    inter = inter && ((bmw[x] >> (c & 31)) & 1u);
+#pragma unroll
+                for (int x = 0; x < NL; ++x) {                                // c-intersection: sorted lists
+                    const bool pend = inter && !(ln[x] & kBmFlag);
+                    const unsigned pw = __ballot_sync(0xffffffffu, pend);
+                    if (pw) {
+                        uint32_t pos = 0;
+                        if (pend) {     // branch-free lower bound from the cursor
+                            const uint32_t* b0 = lb[x];
+                            uint32_t len = ln[x];
+                            while (len > 1) {
+                                const uint32_t half = len >> 1;
+                                b0 = (__ldg(b0 + half - 1) < c) ? b0 + half : b0;
+                                len -= half;
+                            }
+                            inter = len == 1 && __ldg(b0) == c;
+                            pos = (uint32_t)(b0 - lb[x]);
+                        }
+                        // candidates ascend with the lane, so the highest pending lane of
+                        // the virtual warp holds the furthest safe cursor position
+                        const unsigned pv = (pw >> vb) & kGMask;
+                        const int hl = pv ? vb + 31 - __clz(pv) : lane;
+                        const uint32_t mpos = __shfl_sync(0xffffffffu, pos, hl);
+                        if (pv) { lb[x] += mpos; ln[x] -= mpos; }
+                    }
+                }
+                if (count_bytes) bytes += (inter ? 4ull : 0ull) + (inter && ok ? wbytes : 0ull);
+                ok = ok && inter;
+                emit(ok, c);
+            }
             }
         }
     }
@@ -454,7 +496,6 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
         bytes = warp_sum(bytes);
         if (lane == 0) atomicAdd(ctrl + kBytesExt, bytes);
     }
-    (void)vb;
 }
 
 // ---------------------------------------------------------- work donation
