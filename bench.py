@@ -136,6 +136,8 @@ def run_ours(args):
         shuffled level-1 list is cut into world*CHUNKS chunks pulled from a shared
         atomic counter (dynamic root redistribution)."""
         set_q(c, q)
+        if wl.root_range is not None:                 # stated root range (C4)
+            c.set_root_range(*wl.roots(c.level1_size()[0]))
         if world == 1:
             return c.count(wl.mode), [c.stats()]
         _, l1 = c.level1_size()
@@ -252,6 +254,7 @@ def run_ours(args):
         "config": {"workload": wl.name, "description": wl.description, "queries": nq,
                    "graphs": [s.name for s, _ in wl.parts], "embeddings_per_step": step_count,
                    "mode": wl.mode, "l2": "flushed between timed steps (256 MiB write)",
+                   "root_range": (list(wl.root_range) if wl.root_range else None),
                    "parallelism": (f"dynamic root-chunk queue x{world} ({args.chunks_per_rank} chunks/rank/query) + NCCL all-reduce of counts" if world > 1 else "1 GPU")},
         "e2e": {"value": step_count / (e2e_local / 1e3), "unit": "embeddings/s", "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": 8 * nq, "ms_per_step": e2e_local},

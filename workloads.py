@@ -8,7 +8,7 @@ from __future__ import annotations
 
 from dataclasses import dataclass
 
-from inputs import rmat_graph, er_graph, named_query, DENSE5, SPARSE5, dense_family
+from inputs import rmat_graph, rmat_graph_torch, er_graph, named_query, DENSE5, SPARSE5, dense_family
 
 
 @dataclass(frozen=True)
@@ -19,6 +19,10 @@ class GraphSpec:
     def build(self):
         if self.kind == "rmat":
             return rmat_graph(*self.params)
+        if self.kind == "rmat_t":   # same bytes as "rmat" (tests/test_oracle.py), generated with torch
+            import torch
+            *p, seed = self.params
+            return rmat_graph_torch(*p, seed=seed, device="cuda" if torch.cuda.is_available() else "cpu")
         if self.kind == "er":
             return er_graph(*self.params)
         raise KeyError(self.kind)
@@ -34,6 +38,14 @@ class Workload:
     description: str
     parts: tuple          # ((GraphSpec, (Query, ...)), ...)
     mode: str = "hybrid"
+    root_range: tuple | None = None   # (a, b, den): canonical level-1 positions [a*R/den, b*R/den)
+
+    def roots(self, l1: int):
+        """Canonical root range [begin, end) for a level-1 list of size l1."""
+        if self.root_range is None:
+            return 0, l1
+        a, b, den = self.root_range
+        return a * l1 // den, b * l1 // den
 
 
 # configs[0]: triangle and 4-cycle on ER(1000, avg degree 8)
@@ -53,4 +65,24 @@ C2 = Workload(
     "C2", "Dense-5 (11, P:1323-1328) on R-MAT(16,16,.45,.22,.22) + Sparse-5 (8) on R-MAT(16,16,.35,.22,.22); hybrid count",
     ((C2_DENSE_GRAPH, tuple(DENSE5)), (C2_SPARSE_GRAPH, tuple(SPARSE5))))
 
-WORKLOADS = {"C1": C1, "C2": C2}
+# configs[2]: 6-8-vertex dense families on a ~1M-vertex, ~10M-edge power-law graph
+# (com-youtube-like).  Calibrated (profiles/r01_calibration_c3c4.md): R-MAT(20, 10)
+# at a=.50 needs up to 4,600 s for one K8-M query and a=.52 hours; a=.48/.21/.21
+# keeps every one of the 33 queries under 180 s on the first kernel, all counts
+# non-zero and < 2^64.
+C3_GRAPH = GraphSpec("rmat_t", (20, 10, 0.48, 0.21, 0.21, 1))
+C3 = Workload(
+    "C3", "Dense-6/7/8 (33 queries, K_k - M, P:1323-1328) on R-MAT(20,10,.48,.21,.21); hybrid count",
+    ((C3_GRAPH, tuple(dense_family(6) + dense_family(7) + dense_family(8))),))
+
+# configs[3]: 8-vertex dense query on R-MAT scale 22 forcing hybrid BFS/DFS chunking
+# beyond 180 GB.  R-MAT(22, 16, .50, .20, .20): K8's deepest stored level holds
+# ~5.5e11 entries over all roots (4.4 TB of trie) and the full query ~3 h on one
+# GPU; restricted to the first 1/16 of the canonical level-1 list (stated, as
+# SURVEY §8.d allows) the deepest level is still ~3.5e10 entries = 280 GB > 180 GB.
+C4_GRAPH = GraphSpec("rmat_t", (22, 16, 0.50, 0.20, 0.20, 1))
+C4 = Workload(
+    "C4", "K8 on R-MAT(22,16,.50,.20,.20), canonical roots [0, 1/16); hybrid count beyond 180 GB",
+    ((C4_GRAPH, (dense_family(8)[0],)),), root_range=(0, 1, 16))
+
+WORKLOADS = {"C1": C1, "C2": C2, "C3": C3, "C4": C4}
