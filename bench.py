@@ -35,6 +35,9 @@ def _args():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--chunks-per-rank", type=int, default=16, help="dynamic root queue granularity (N > 1)")
+    ap.add_argument("--donate", action="store_true",
+                    help="N > 1: add Alg. 3 prefix donations (NCCL send/recv) to the root queue; validated with "
+                         "gloo and two ranks on one GPU only, so off by default")
     ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     return ap.parse_args()
 
@@ -126,6 +129,7 @@ def run_ours(args):
     from paper_conf_sc_xiangkshs21_b200 import dist as D
     store = D.default_store() if world > 1 else None
     pass_id = [0]
+    donations = [0]
 
     def set_q(c, q):
         qr, qc = q.csr()
@@ -143,6 +147,13 @@ def run_ours(args):
         _, l1 = c.level1_size()
         cs = max(1, -(-l1 // (world * args.chunks_per_rank)))
         queue = D.RootQueue(store, f"{tag}", D.n_chunks(l1, cs))
+        if args.donate:
+            # root chunks, then serve as a receiver of donated flat prefixes (Alg. 3)
+            eng = D.CutsEngine(c, wl.mode)
+            ws = D.WorkSharing(store, f"ws{tag}", rank, world, eng, transport_device=dev)
+            local = ws.run(queue, cs)
+            donations[0] += ws.sent
+            return local, eng.stats
         local, sts = 0, []
         while (ch := queue.next()) is not None:
             b, e = D.chunk_bounds(ch, cs)
@@ -255,7 +266,10 @@ def run_ours(args):
                    "graphs": [s.name for s, _ in wl.parts], "embeddings_per_step": step_count,
                    "mode": wl.mode, "l2": "flushed between timed steps (256 MiB write)",
                    "root_range": (list(wl.root_range) if wl.root_range else None),
-                   "parallelism": (f"dynamic root-chunk queue x{world} ({args.chunks_per_rank} chunks/rank/query) + NCCL all-reduce of counts" if world > 1 else "1 GPU")},
+                   "parallelism": (f"dynamic root-chunk queue x{world} ({args.chunks_per_rank} chunks/rank/query)"
+                                   + (" + Alg. 3 prefix donations (NCCL send/recv)" if args.donate else "")
+                                   + " + NCCL all-reduce of counts" if world > 1 else "1 GPU"),
+                   "donations": donations[0] if world > 1 else 0},
         "e2e": {"value": step_count / (e2e_local / 1e3), "unit": "embeddings/s", "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": 8 * nq, "ms_per_step": e2e_local},
         "gpu_launches": launches // args.steps,

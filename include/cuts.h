@@ -95,6 +95,10 @@ typedef struct {
 /* debug / instrumentation flags for cuts_set_debug */
 #define CUTS_DEBUG_TIMING 1u   /* CUDA events around each kernel -> ms_extend / ms_plan     */
 #define CUTS_DEBUG_BYTES  2u   /* per-warp algorithmic byte counters (perturbs timing)      */
+#define CUTS_DEBUG_NO_REUSE 4u /* HYBRID: disable the ancestor-set source (ablation); BFS
+                                  mode never uses it                                        */
+#define CUTS_DEBUG_NO_PACK  8u /* at the next cuts_load_graph: no packed (id | degree) copy
+                                  of col in the arena (ablation)                            */
 
 /* Create a context bound to opts->device / opts->stream / opts->arena.
  * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */

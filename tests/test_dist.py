@@ -126,3 +126,15 @@ def test_gloo_work_sharing_donations(world):
     assert sum(r["local"] for r in res) == serial
     assert sum(r["sent"] for r in res) >= 1
     assert sum(r["sent"] for r in res) == sum(r["recv"] for r in res)
+
+
+def test_workload_root_ranges():
+    """The stated root range of C4 (first 1/16 of the canonical level-1 list) and
+    the full range of the other configs."""
+    from workloads import WORKLOADS
+    assert WORKLOADS["C4"].roots(1600) == (0, 100)
+    assert WORKLOADS["C4"].roots(17) == (0, 1)
+    for name in ("C1", "C2", "C3"):
+        assert WORKLOADS[name].roots(1234) == (0, 1234)
+    assert len(WORKLOADS["C3"].parts[0][1]) == 33
+    assert WORKLOADS["C4"].parts[0][1][0].name == "K8"

@@ -23,6 +23,15 @@ pytestmark = pytest.mark.gpu
 
 
 @pytest.fixture(scope="module")
+def cuts():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_xiangkshs21_b200 import Cuts
+    return Cuts
+
+
+@pytest.fixture(scope="module")
 def bench_ctx():
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
@@ -86,3 +95,65 @@ def test_c2_full_size_closed_forms(bench_ctx, part):
         want = _falling(d, s)
         got = bench_ctx.count("hybrid")
         assert got == want, (spec.name, name, got, want)
+
+
+def _hub_ranges(g, q, ranks):
+    """[pos, pos+1) of the roots ranked `ranks` by degree in the canonical level-1 list."""
+    d = g.degrees()
+    canon = np.nonzero(d >= max(q.degrees()))[0]
+    order = np.argsort(-d[canon], kind="stable")
+    return [(int(order[r]), int(order[r]) + 1) for r in ranks if r < len(order)]
+
+
+def test_c3_full_size_root_samples(bench_ctx):
+    """configs[2] at full size: 9 of the 33 Dense-6/7/8 queries, on the root ranked
+    2000th by degree (the cliques live among high-degree vertices; the oracle takes
+    minutes on the top hubs) and two evenly spaced roots."""
+    wl = WORKLOADS["C3"]
+    spec, qs = wl.parts[0]
+    g = spec.build()
+    bench_ctx.load_csr(g, validate=True)
+    nonzero = 0
+    for q in qs[::4]:
+        _set(bench_ctx, q)
+        l1, _ = bench_ctx.level1_size()
+        for a, b in _hub_ranges(g, q, (2000,)) + _ranges(l1, 1, 2):
+            bench_ctx.set_root_range(a, b)
+            got = bench_ctx.count(wl.mode)
+            want = oracle.count(g, q, root_begin=a, root_end=b)
+            assert got == want, (q.name, a, b, got, want)
+            nonzero += want > 0
+        bench_ctx.set_root_range()
+    assert nonzero >= 5
+
+
+def test_c4_root_samples_and_chunk_invariance(cuts):
+    """configs[3] graph: oracle parity on sampled roots inside the stated range, and
+    the count + per-level sizes of one hub root identical at three arena sizes
+    (the smaller arenas force many more DFS chunks)."""
+    wl = WORKLOADS["C4"]
+    spec, (q,) = wl.parts[0]
+    g = spec.build()
+    qr, qc = q.csr()
+    res = []
+    for arena in (None, 512 << 20, 160 << 20):
+        ctx = cuts(device=0, arena_bytes=arena)
+        ctx.load_csr(g, validate=arena is None)
+        ctx.set_query(qr, qc)
+        l1, _ = ctx.level1_size()
+        b0, b1 = wl.roots(l1)
+        if arena is None:
+            for a, b in [r for r in _hub_ranges(g, q, (6000,)) if b0 <= r[0] < b1] + [(b0, b0 + 1), (b1 - 1, b1)]:
+                ctx.set_root_range(a, b)
+                got = ctx.count("hybrid")
+                assert got == oracle.count(g, q, root_begin=a, root_end=b), (a, b)
+        a, b = _hub_ranges(g, q, (300,))[0]
+        ctx.set_root_range(a, b)
+        cnt = ctx.count("hybrid")
+        st = ctx.stats()
+        res.append((cnt, st["level_size"], st["chunks"]))
+        ctx.close()
+        del ctx
+    assert res[0][0] == res[1][0] == res[2][0]
+    assert res[0][1] == res[1][1] == res[2][1]
+    assert res[2][2] > res[0][2]

@@ -99,6 +99,50 @@ def test_chunk_invariance(cuts, arena_kib):
         assert c.stats()["level_size"] == lv
 
 
+@pytest.mark.parametrize("arena_kib", [64, 128, 512, 4096])
+def test_ancestor_reuse_chunked(cuts, arena_kib):
+    """HYBRID's ancestor-set source (ordered levels, entry-aligned chunks and the
+    oversized-entry fallback at tiny arenas) against the oracle and against the
+    same run with the reuse disabled (CUTS_DEBUG_NO_REUSE)."""
+    g = rmat_graph(8, 6, a=0.5, b=0.2, c=0.2, seed=3)
+    c = cuts(device=0, arena_bytes=arena_kib << 10)
+    c.load_csr(g)
+    for q in [DENSE5[0], DENSE5[3], DENSE5[5]] + dense_family(6)[::3] + dense_family(7)[::4] + dense_family(8)[::5]:
+        want, lv = oracle.count(g, q, levels=True)
+        _set(c, q)
+        for flags in (0, 4):
+            c.lib.cuts_set_debug(c.h, flags)
+            assert c.count("hybrid") == want, (arena_kib, q.name, flags)
+            assert c.stats()["level_size"] == lv, (arena_kib, q.name, flags)
+        c.set_debug()
+
+
+def test_packed_degree_stream_ablation(cuts):
+    """The packed (id | min(deg,31)) candidate stream against the plain col + deg
+    gather (CUTS_DEBUG_NO_PACK at load): same counts and level sizes, incl. degree
+    thresholds above 1 and hubs with degree >= 31."""
+    g = rmat_graph(8, 5, a=0.55, b=0.2, c=0.2, seed=4)
+    assert g.degrees().max() > 31
+    c = cuts(device=0, arena_bytes=64 << 20)
+    for flags in (0, 8):
+        c.lib.cuts_set_debug(c.h, flags)
+        c.load_csr(g)
+        for q in (DENSE5[9], DENSE5[10], SPARSE5[1], SPARSE5[4], named_query("C4"), dense_family(6)[5]):
+            want, lv = oracle.count(g, q, levels=True)
+            _set(c, q)
+            for mode in ("hybrid", "bfs"):
+                assert c.count(mode) == want, (flags, q.name, mode)
+                assert c.stats()["level_size"] == lv, (flags, q.name, mode)
+    c.set_debug()
+
+
+def test_ancestor_reuse_enumerate(ctx):
+    g = er_graph(40, 420, 7)
+    ctx.load_csr(g)
+    for q in [DENSE5[0]] + dense_family(6)[:4] + dense_family(7)[:2]:
+        _check_full(ctx, g, q, modes=("hybrid",))
+
+
 # ------------------------------------------------------------ 5-vertex family
 @pytest.mark.parametrize("seed", [2, 3])
 def test_5vertex_families_rmat9(ctx, seed):
