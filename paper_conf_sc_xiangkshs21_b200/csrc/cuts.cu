@@ -56,6 +56,7 @@ struct cuts_ctx {
     uint32_t* deg = nullptr;
     uint32_t* hub = nullptr;               // hub[v] -> bitmap row, or kNoHub
     uint32_t* bm = nullptr;                // hub bitmaps
+    uint32_t* colx = nullptr;              // packed (id | min(deg,31) << 27) copy of col, or null
     uint32_t words = 0;
     uint64_t nhubs = 0, hub_t_used = 0;
     uint32_t hub_t = 0;                    // requested threshold (0 auto, UINT32_MAX off)
@@ -82,6 +83,13 @@ struct cuts_ctx {
     cuts_poll_fn poll = nullptr;
     cuts_ship_fn ship = nullptr;
     void* user = nullptr;
+    // ancestor-set reuse: anc[J] = ancestor level whose children range
+    // sources level J's candidates (0: none); bit a of need_ord: level a -> a+1 is
+    // written ordered (children contiguous per parent, exact offsets kept)
+    uint32_t anc[kMaxK + 1] = {};
+    uint32_t need_ord = 0;
+    struct OrdState { const uint64_t* cpos; uint64_t w0; uint64_t ea; const uint2* lv; bool valid; };
+    OrdState ord[kMaxK + 1] = {};
     uint64_t dfs_next[kMaxK + 1] = {};   // first entry of level d not yet planned
     uint64_t dfs_end[kMaxK + 1] = {};    // end of level d's entries still owned here
     bool dfs_on[kMaxK + 1] = {};
@@ -227,6 +235,11 @@ struct Window {
     uint64_t* src;
     uint64_t* lst_off;   // (J-1) x W list descriptors from k_plan
     uint32_t* lst_len;
+    uint64_t* cpos;      // ordered levels: exclusive scan of the children per entry (W+1)
+    Reuse ru{};          // ancestor-set source for this level (ru.a == 0: off)
+    uint64_t* ord_cnt = nullptr;         // pass A output (children per entry)
+    const uint64_t* ord_pos = nullptr;   // pass B: exact child offsets
+    uint32_t ord_ea = 0;                 // pass B: first entry of the chunk
     uint64_t* ub;
     uint64_t* offs;
     void* cub_tmp;
@@ -237,7 +250,7 @@ struct Window {
 template <int J>
 void launch_plan_t(cuts_ctx* ctx, const Graph& g, const Trie& t, const Window& w, int grid) {
     k_plan<J><<<grid, 256, 0, ctx->stream>>>(g, t, ctx->q, w.w0, w.W, w.path, w.src, w.ub, w.lst_off, w.lst_len, ctx->ctrl,
-                                             (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0);
+                                             (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0, w.ru);
 }
 
 void launch_plan(cuts_ctx* ctx, int J, const Graph& g, const Trie& t, const Window& w) {
@@ -270,7 +283,9 @@ void launch_extend_g(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0
     k_extend<J, NL, M, G><<<(unsigned)grid, 256, 0, ctx->stream>>>(g, ctx->q, w.w0, w.W, w.path, w.src, w.offs,
                                                                    w.lst_off, w.lst_len, t0, t1,
                                                                    out_level, out_rows, cap, ctx->ctrl,
-                                                                   (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0, batch);
+                                                                   (ctx->debug & CUTS_DEBUG_BYTES) && !w.ord_cnt ? 1 : 0, batch,
+                                                                   w.ru.a ? ctx->q.qdeg[w.ru.a] : 0u,
+                                                                   w.ru.lv, w.ord_cnt, w.ord_pos, w.ord_ea);
 }
 
 template <int J, int NL, int M>
@@ -326,8 +341,8 @@ struct Run {
 
 uint64_t window_scratch_bytes(uint64_t W, int J, size_t cub_bytes) {
     const uint64_t nl = (uint64_t)std::max(J - 1, 1);
-    return align_up((uint64_t)J * W * 4) + align_up(W * 8) + 2 * align_up((W + 1) * 8) + align_up(nl * W * 8) +
-           align_up(nl * W * 4) + align_up(cub_bytes) + 6 * kAlign;
+    return align_up((uint64_t)J * W * 4) + align_up(W * 8) + 3 * align_up((W + 1) * 8) + align_up(nl * W * 8) +
+           align_up(nl * W * 4) + align_up(cub_bytes) + 7 * kAlign;
 }
 
 cuts_status read_ctrl(cuts_ctx* ctx) {
@@ -390,6 +405,7 @@ cuts_status alloc_window(cuts_ctx* ctx, int J, uint64_t W, Window* w) {
     const uint64_t nl = (uint64_t)std::max(J - 1, 1);
     w->lst_off = (uint64_t*)p; p += align_up(nl * W * 8);
     w->lst_len = (uint32_t*)p; p += align_up(nl * W * 4);
+    w->cpos = (uint64_t*)p; p += align_up((W + 1) * 8);
     w->cub_tmp = p;
     w->cub_bytes = cub_bytes;
     return CUTS_OK;
@@ -397,7 +413,7 @@ cuts_status alloc_window(cuts_ctx* ctx, int J, uint64_t W, Window* w) {
 
 // window size for depth J: bounded so all depths' scratch takes <= 1/8 of the arena
 uint64_t pick_window(cuts_ctx* ctx, uint64_t N) {
-    uint64_t per = (uint64_t)(ctx->q.k) * 4 + 24 + (uint64_t)std::max<int>((int)ctx->q.k - 2, 1) * 12;   // path + src + ub + offs + list descriptors
+    uint64_t per = (uint64_t)(ctx->q.k) * 4 + 32 + (uint64_t)std::max<int>((int)ctx->q.k - 2, 1) * 12;   // path + src + ub + offs + cpos + list descriptors
     uint64_t budget = ctx->arena_bytes / 8 / std::max<uint32_t>(1, ctx->q.k - 1);
     uint64_t w = budget / per;
     w = std::max<uint64_t>(w, 1);
@@ -454,10 +470,113 @@ cuts_status maybe_donate(cuts_ctx* ctx, Run& r) {
 }
 
 // HYBRID: process entries [0, N) of level J stored at r.t.lv[J] (DFS over chunks)
+inline bool reuse_on(const cuts_ctx* ctx, const Run& r) {
+    return r.mode == CUTS_HYBRID && !(ctx->debug & CUTS_DEBUG_NO_REUSE);
+}
+
+// level J+1's chunk share of the free space: deeper stored levels (J+2 .. k-1)
+// and their window scratch share the rest
+cuts_status chunk_cap(cuts_ctx* ctx, int J, uint64_t* cap) {
+    const int k = (int)ctx->q.k;
+    uint64_t deeper_scratch = 0;
+    const uint64_t wd = pick_window(ctx, ~0ull);
+    size_t cb = 0;
+    CK(cub::DeviceScan::ExclusiveSum(nullptr, cb, (uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)wd + 1, ctx->stream));
+    for (int d = J + 1; d <= k - 1; ++d) deeper_scratch += window_scratch_bytes(wd, d, cb);
+    const uint64_t fb = free_bytes(ctx);
+    const uint64_t avail = fb > deeper_scratch ? fb - deeper_scratch : 0;
+    const uint64_t share = avail / (uint64_t)(k - 1 - J);
+    *cap = std::min<uint64_t>(share / sizeof(uint2), kMaxLevel);
+    if (*cap == 0) return fail(ctx, CUTS_ENOMEM, "HYBRID: arena too small for level %d (free %llu B)", J + 1, (unsigned long long)fb);
+    return CUTS_OK;
+}
+
+cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N);
+
+// unordered chunks over items [i0, i1) of window w (children bounded by ub)
+cuts_status hybrid_items(cuts_ctx* ctx, Run& r, int J, const Window& w, uint64_t i0, uint64_t i1) {
+    for (uint64_t t = i0; t < i1;) {
+        uint64_t cap;
+        TRY(chunk_cap(ctx, J, &cap));
+        uint64_t t1 = std::min<uint64_t>(i1, t + cap);   // items bound children (ub)
+        uint64_t off;
+        const uint64_t bot_save = ctx->bot;
+        TRY(alloc_bot(ctx, (t1 - t) * sizeof(uint2), &off));
+        uint2* out = (uint2*)(ctx->arena + off);
+        CK(cudaMemsetAsync(ctx->ctrl + kCursor, 0, sizeof(unsigned long long), ctx->stream));
+        TRY(extend_range(ctx, r, J, w, t, t1, kWrite, out, t1 - t));
+        CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        uint64_t size = ctx->h_ctrl[kCursor];
+        if (size > t1 - t) return fail(ctx, CUTS_ENOMEM, "internal: chunk overflow");
+        ctx->st.level_size[J + 1] += size;
+        ctx->bot = off + size * sizeof(uint2);     // shrink to the exact level size
+        if (size) {
+            r.t.lv[J + 1] = out;
+            TRY(hybrid_level(ctx, r, J + 1, size));
+        }
+        ctx->bot = bot_save;
+        t = t1;
+        if (t < i1) TRY(maybe_donate(ctx, r));
+    }
+    return CUTS_OK;
+}
+
+// ordered chunks (level J+1 feeds an ancestor-set source deeper down): pass A
+// counts each entry's children, a scan gives their exact offsets, chunks are cut
+// at entry boundaries so each chunk holds whole sibling ranges, pass B writes
+// every entry's children contiguously (no atomics).
+cuts_status hybrid_ordered(cuts_ctx* ctx, Run& r, int J, Window& w) {
+    CK(cudaMemsetAsync(w.ub, 0, (w.W + 1) * sizeof(uint64_t), ctx->stream));
+    Window wa = w;
+    wa.ord_cnt = w.ub;
+    TRY(extend_range(ctx, r, J, wa, 0, w.total, kCount, nullptr, 0));
+    CK(cub::DeviceScan::ExclusiveSum(w.cub_tmp, w.cub_bytes, w.ub, w.cpos, (int64_t)w.W + 1, ctx->stream));
+    ctx->st.launches += 2;
+    for (uint32_t ea = 0; ea < w.W;) {
+        uint64_t cap;
+        TRY(chunk_cap(ctx, J, &cap));
+        k_find_chunk<<<1, 1, 0, ctx->stream>>>(w.cpos, w.offs, w.W, ea, cap, ctx->ctrl + kFind);
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(ctx->h_ctrl + kFind, ctx->ctrl + kFind, 5 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        ctx->st.launches++;
+        const uint32_t eb = (uint32_t)ctx->h_ctrl[kFind];
+        const uint64_t size = ctx->h_ctrl[kFind + 1], i0 = ctx->h_ctrl[kFind + 2], i1 = ctx->h_ctrl[kFind + 3];
+        if (eb > ea) {
+            const uint64_t bot_save = ctx->bot;
+            uint64_t off;
+            TRY(alloc_bot(ctx, std::max<uint64_t>(size, 1) * sizeof(uint2), &off));
+            uint2* out = (uint2*)(ctx->arena + off);
+            if (size) {
+                Window wb = w;
+                wb.ord_pos = w.cpos;
+                wb.ord_ea = ea;
+                TRY(extend_range(ctx, r, J, wb, i0, i1, kWrite, out, size));
+                ctx->st.level_size[J + 1] += size;
+                ctx->ord[J] = {w.cpos, w.w0, ea, out, true};
+                r.t.lv[J + 1] = out;
+                TRY(hybrid_level(ctx, r, J + 1, size));
+                ctx->ord[J].valid = false;
+            }
+            ctx->bot = bot_save;
+            ea = eb;
+        } else {
+            // one entry whose children exceed the share: unordered item pieces; its
+            // subtree gets no ancestor-set source from level J
+            TRY(hybrid_items(ctx, r, J, w, i0, ctx->h_ctrl[kFind + 4]));
+            ea += 1;
+        }
+        if (ea < w.W) TRY(maybe_donate(ctx, r));
+    }
+    return CUTS_OK;
+}
+
 cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     const int k = (int)ctx->q.k;
     const bool last = (J == k - 1);
     const uint64_t top_save = ctx->top;
+    const bool ordered = !last && reuse_on(ctx, r) && ((ctx->need_ord >> J) & 1u);
     ctx->dfs_on[J] = true;
     ctx->dfs_next[J] = 0;
     ctx->dfs_end[J] = N;
@@ -469,45 +588,17 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
         w.w0 = w0;
         w.W = (uint32_t)std::min<uint64_t>(pick_window(ctx, N), N - w0);
         ctx->dfs_next[J] = w0 + w.W;
+        const uint32_t a = ctx->anc[J];
+        if (a && reuse_on(ctx, r) && ctx->ord[a].valid)
+            w.ru = Reuse{ctx->ord[a].lv, ctx->ord[a].cpos, ctx->ord[a].w0, ctx->ord[a].ea, a, ctx->q.bw[a]};
         TRY(alloc_window(ctx, J, w.W, &w));
         TRY(plan_window(ctx, r, J, w));
         if (last) {
             TRY(extend_range(ctx, r, J, w, 0, w.total, r.enumerate ? kEnum : kCount, nullptr, 0));
+        } else if (ordered) {
+            TRY(hybrid_ordered(ctx, r, J, w));
         } else {
-            for (uint64_t t = 0; t < w.total;) {
-                // L_{J+1} chunk takes its share of the free space; deeper stored levels
-                // (J+2 .. k-1) and their window scratch share the rest.
-                uint64_t deeper_scratch = 0;
-                const uint64_t wd = pick_window(ctx, ~0ull);
-                size_t cb = 0;
-                CK(cub::DeviceScan::ExclusiveSum(nullptr, cb, (uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)wd + 1, ctx->stream));
-                for (int d = J + 1; d <= k - 1; ++d) deeper_scratch += window_scratch_bytes(wd, d, cb);
-                uint64_t fb = free_bytes(ctx);
-                uint64_t avail = fb > deeper_scratch ? fb - deeper_scratch : 0;
-                uint64_t share = avail / (uint64_t)(k - 1 - J);
-                uint64_t cap = std::min<uint64_t>(share / sizeof(uint2), kMaxLevel);
-                if (cap == 0) return fail(ctx, CUTS_ENOMEM, "HYBRID: arena too small for level %d (free %llu B)", J + 1, (unsigned long long)fb);
-                uint64_t t1 = std::min<uint64_t>(w.total, t + cap);   // items bound children (ub)
-                uint64_t off;
-                const uint64_t bot_save = ctx->bot;
-                TRY(alloc_bot(ctx, (t1 - t) * sizeof(uint2), &off));
-                uint2* out = (uint2*)(ctx->arena + off);
-                CK(cudaMemsetAsync(ctx->ctrl + kCursor, 0, sizeof(unsigned long long), ctx->stream));
-                TRY(extend_range(ctx, r, J, w, t, t1, kWrite, out, t1 - t));
-                CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
-                CK(cudaStreamSynchronize(ctx->stream));
-                uint64_t size = ctx->h_ctrl[kCursor];
-                if (size > t1 - t) return fail(ctx, CUTS_ENOMEM, "internal: chunk overflow");
-                ctx->st.level_size[J + 1] += size;
-                ctx->bot = off + size * sizeof(uint2);     // shrink to the exact level size
-                if (size) {
-                    r.t.lv[J + 1] = out;
-                    TRY(hybrid_level(ctx, r, J + 1, size));
-                }
-                ctx->bot = bot_save;
-                t = t1;
-                if (t < w.total) TRY(maybe_donate(ctx, r));
-            }
+            TRY(hybrid_items(ctx, r, J, w, 0, w.total));
         }
         ctx->top = top_save;
         w0 += w.W;
@@ -540,6 +631,14 @@ cuts_status bfs_levels(cuts_ctx* ctx, Run& r, int J0, uint64_t N1) {
             w.W = (uint32_t)std::min<uint64_t>(W, N - w0);
             TRY(plan_window(ctx, r, J, w));
             TRY(extend_range(ctx, r, J, w, 0, w.total, last ? (r.enumerate ? kEnum : kCount) : kWrite, out, cap));
+            if (!last && w0 + W < N) {     // stop at the first window that overflows the level
+                CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
+                CK(cudaStreamSynchronize(ctx->stream));
+                if (ctx->h_ctrl[kCursor] > cap)
+                    return fail(ctx, CUTS_ENOMEM, "BFS: level %d exceeds the room for %llu entries after %llu of %llu "
+                                "entries of level %d (use CUTS_HYBRID)", J + 1, (unsigned long long)cap,
+                                (unsigned long long)(w0 + W), (unsigned long long)N, J);
+            }
         }
         if (!last) {
             CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
@@ -708,10 +807,10 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     r.enumerate = enumerate;
     r.rows = rows;
     r.cap_rows = cap_rows;
-    r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words};
+    r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words, ctx->colx};
     uint64_t n1 = 0;
     const int k = (int)ctx->q.k;
-    for (int j = 0; j <= kMaxK; ++j) { ctx->dfs_on[j] = false; ctx->dfs_next[j] = ctx->dfs_end[j] = 0; }
+    for (int j = 0; j <= kMaxK; ++j) { ctx->dfs_on[j] = false; ctx->dfs_next[j] = ctx->dfs_end[j] = 0; ctx->ord[j].valid = false; }
     if (ctx->pre_j) {
         TRY(build_prefix_levels(ctx, r));
         const int J0 = (int)ctx->pre_j;
@@ -845,7 +944,7 @@ cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint6
                                                     (unsigned long long)ends[0], (unsigned long long)ends[1], (unsigned long long)nnz);
     if (validate && n) {
         CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
-        Graph g{d_row_ptr, d_col, ctx->deg, nullptr, nullptr, n, 0};
+        Graph g{d_row_ptr, d_col, ctx->deg, nullptr, nullptr, n, 0, nullptr};
         unsigned grid = (unsigned)std::min<uint64_t>(((uint64_t)n * 32 + 255) / 256, (uint64_t)ctx->num_sms * 16);
         k_validate<<<grid, 256, 0, ctx->stream>>>(g, ctx->ctrl);
         CK(cudaGetLastError());
@@ -853,6 +952,17 @@ cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint6
         if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_EINVAL, "graph is not canonical symmetric CSR (sorted, no loops/dups, ids < n)");
     }
     TRY(build_hubs(ctx));
+    // packed candidate stream (degree filter without a gather) when ids fit 27 bits
+    ctx->colx = nullptr;
+    const uint64_t colx_bytes = align_up(nnz * 4);
+    if (nnz && n <= kPackMask && ctx->base_off + colx_bytes + (ctx->arena_bytes / 2) <= ctx->arena_bytes &&
+        !(ctx->debug & CUTS_DEBUG_NO_PACK)) {
+        ctx->colx = (uint32_t*)(ctx->arena + ctx->base_off);
+        unsigned grid = (unsigned)std::min<uint64_t>((nnz + 255) / 256, (uint64_t)ctx->num_sms * 16);
+        k_pack<<<grid, 256, 0, ctx->stream>>>(d_col, nnz, ctx->deg, ctx->colx);
+        CK(cudaGetLastError());
+        ctx->base_off += colx_bytes;
+    }
     ctx->has_graph = true;
     return CUTS_OK;
 }
@@ -872,6 +982,17 @@ cuts_status cuts_set_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr, c
     ctx->has_query = false;
     TRY(plan_query(ctx, k, row_ptr, col, order, &qp));
     ctx->q = qp;
+    // ancestor-set reuse plan: deepest a in [2, J-1] with |bw[a]| >= 2 (an actual
+    // intersection), bw[a] a subset of bw[J] and deg_Q(S[a]) <= deg_Q(S[J])
+    ctx->need_ord = 0;
+    for (uint32_t J = 0; J <= kMaxK; ++J) ctx->anc[J] = 0;
+    for (uint32_t J = 3; J < qp.k; ++J)
+        for (uint32_t a = J - 1; a >= 2; --a)
+            if (__builtin_popcount(qp.bw[a]) >= 2 && (qp.bw[a] & ~qp.bw[J]) == 0 && qp.qdeg[a] <= qp.qdeg[J]) {
+                ctx->anc[J] = a;
+                ctx->need_ord |= 1u << a;
+                break;
+            }
     ctx->root_begin = 0;
     ctx->root_end = ~0ull;
     ctx->slice_begin = 0;

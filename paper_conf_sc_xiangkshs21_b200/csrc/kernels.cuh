@@ -34,6 +34,25 @@ struct Trie {                  // lv[l] = level l (1-based): .x = data vertex, .
     const uint2* lv[kMaxK];
 };
 
+// Ancestor-set reuse ("incremental intersection").  Level a+1 was
+// written ORDERED: the children of level-a entry x are the contiguous range
+// [cpos[x-w0] - cpos[ea], cpos[x-w0+1] - cpos[ea]) of the level-(a+1) chunk
+// lv, and their vertices are exactly {c in the intersection of N(f(S[p])),
+// p in bw[a] : deg(c) >= qdeg[a], c not on x's path}.  When bw[a] is a subset
+// of bw[J] and qdeg[a] <= qdeg[J], that range contains every candidate of a
+// level-J descendant of x, so it can replace the lists of bw[a] as the source.
+struct Reuse {
+    const uint2* lv;           // level a+1 chunk (candidate source for trie-sourced entries)
+    const uint64_t* cpos;      // level a window's exclusive scan of child counts
+    uint64_t w0;               // level a window start
+    uint64_t ea;               // first level-a entry (window-relative) of the level a+1 chunk
+    uint32_t a;                // ancestor level (0: off)
+    uint32_t bwa;              // bw[a]
+};
+
+constexpr uint64_t kTrieSrc = 1ull << 63;   // src_off flag: the source is a trie range
+constexpr uint32_t kSkip = 0xffffffffu;     // list-slot length: no list in this slot
+
 struct Graph {
     const uint64_t* __restrict__ row_ptr;
     const uint32_t* __restrict__ col;
@@ -42,16 +61,19 @@ struct Graph {
     const uint32_t* __restrict__ bm;    // hub adjacency bitmaps, words u32 per row
     uint32_t n;
     uint32_t words;
+    const uint32_t* __restrict__ colx;  // col with min(deg, 31) packed in bits 27..31 (nullptr: n >= 2^27)
 };
 
 constexpr uint32_t kNoHub = 0xffffffffu;
+constexpr int kPackShift = 27;               // colx: vertex id in bits 0..26, min(deg, 31) above
+constexpr uint32_t kPackMask = (1u << kPackShift) - 1u;
 constexpr uint32_t kBmFlag = 0x80000000u;   // list-slot length flag: probe a bitmap instead
 
 enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 
 // control block (u64 words in the arena)
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
-            kEnumCursor = 6, kNumSel = 7, kWork = 8, kCtrlWords = 64 };
+            kEnumCursor = 6, kNumSel = 7, kWork = 8, kFind = 24, kCtrlWords = 64 };
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
     if (v == 0) return;
@@ -83,6 +105,16 @@ __device__ __forceinline__ bool list_contains(const uint32_t* __restrict__ col, 
 __global__ void k_degree(const uint64_t* __restrict__ row_ptr, uint32_t n, uint32_t* __restrict__ deg) {
     for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x)
         deg[v] = (uint32_t)(row_ptr[v + 1] - row_ptr[v]);
+}
+
+// colx[p] = col[p] | min(deg(col[p]), 31) << 27: the candidate stream carries the
+// degree-filter input (Def. 5), so the filter costs no random 4 B gather
+__global__ void k_pack(const uint32_t* __restrict__ col, uint64_t nnz, const uint32_t* __restrict__ deg,
+                       uint32_t* __restrict__ colx) {
+    for (uint64_t p = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; p < nnz; p += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t u = col[p];
+        colx[p] = u | (min(deg[u], 31u) << kPackShift);
+    }
 }
 
 // SV-style membership rows (Alg. 2 l.7-17's |V|-sized scatter vector, P:1055-1072,
@@ -210,7 +242,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                                               uint64_t* __restrict__ ub,
                                               uint64_t* __restrict__ lst_off,
                                               uint32_t* __restrict__ lst_len,
-                                              unsigned long long* __restrict__ ctrl, int count_bytes) {
+                                              unsigned long long* __restrict__ ctrl, int count_bytes, Reuse ru) {
     const uint32_t bw = q.bw[J];
     unsigned long long bytes_plan = 0, bytes_ext = 0;
     for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e <= W; e += gridDim.x * blockDim.x) {
@@ -219,8 +251,10 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         uint2 cur = t.lv[J][w0 + e];
         path[J - 1] = cur.x;
         uint32_t idx = cur.y;
+        uint32_t xa = 0;                             // index of the level-a ancestor (reuse)
 #pragma unroll
         for (int p = J - 2; p >= 0; --p) {          // trie walk
+            if (p + 1 == (int)ru.a) xa = idx;
             cur = t.lv[p + 1][idx];
             path[p] = cur.x;
             idx = cur.y;
@@ -243,13 +277,36 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                 if (best < 0 || d < best_d) { best = p; best_d = d; best_b = b; }
             }
         }
-        src_off[e] = best_b;
-        ub[e] = best_d;
+        // ancestor-set source: the children range of the level-a ancestor replaces
+        // the lists of bw[a] when it is no longer than every remaining list
+        uint32_t keep = bw;                          // lists still to be tested
+        bool trie = false;
+        uint64_t trie_off = 0, rest_sum = 0;
+        uint32_t trie_len = 0;
+        if (ru.a) {
+            const uint64_t k0 = (uint64_t)xa - ru.w0;
+            const uint64_t c0 = ru.cpos[k0], base = ru.cpos[ru.ea];
+            trie_len = (uint32_t)(ru.cpos[k0 + 1] - c0);
+            trie_off = c0 - base;
+            uint32_t rest_min = 0xffffffffu;
+#pragma unroll
+            for (int p = 0; p < J; ++p)
+                if (((bw & ~ru.bwa) >> p) & 1u) { rest_min = min(rest_min, ln_[p]); rest_sum += ln_[p]; }
+            if (trie_len <= rest_min) { trie = true; keep = bw & ~ru.bwa; }
+        }
+        if (trie) {
+            src_off[e] = trie_off | kTrieSrc;
+            ub[e] = trie_len;
+            best = -1;
+        } else {
+            src_off[e] = best_b;
+            ub[e] = best_d;
+        }
         // other lists: hub rows become bitmap probes; then sort by length
         int x = 0;
 #pragma unroll
         for (int p = 0; p < J; ++p) {
-            if (p != best && ((bw >> p) & 1u)) {
+            if (p != best && ((keep >> p) & 1u)) {
                 const uint32_t h = g.hub ? __ldg(g.hub + path[p]) : kNoHub;
                 if (h != kNoHub) { lb_[p] = (uint64_t)h * g.words; ln_[p] |= kBmFlag; }
             } else {
@@ -276,7 +333,11 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         for (int p = 0; p < J; ++p) path_s[(size_t)p * W + e] = path[p];
         if (count_bytes) {   // 8 (entry) + 8(J-1) (hops) + 16 per list bound
             bytes_plan += 8ull + 8ull * (J - 1) + 16ull * __popc(bw);
-            bytes_ext += 4ull * lists;                   // every backward list read once
+            if (trie) {          // the ancestor range (8 B entries) + the lists not covered by it
+                bytes_ext += 8ull * trie_len + 4ull * rest_sum;
+            } else {
+                bytes_ext += 4ull * lists;               // every backward list read once
+            }
         }
     }
     if (count_bytes) {
@@ -319,7 +380,9 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                                                uint2* __restrict__ out_level,
                                                uint32_t* __restrict__ out_rows, uint64_t cap,
                                                unsigned long long* __restrict__ ctrl, int count_bytes,
-                                               uint32_t batch) {
+                                               uint32_t batch, uint32_t qda, const uint2* __restrict__ rsrc,
+                                               uint64_t* __restrict__ ord_cnt,
+                                               const uint64_t* __restrict__ ord_pos, uint32_t ord_ea) {
     constexpr int VPW = 32 / G;
     constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
     constexpr int NLA = NL > 0 ? NL : 1;
@@ -359,7 +422,7 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
             const uint32_t e = ea + (has ? ei : 0);
             // this entry's item range, clipped to [t0, t1)
             uint32_t ilo = 0, ihi = 0;
-            uint64_t so = 0;
+            uint64_t so = 0, obase = 0;
             uint32_t path[J];
             const uint32_t* lb[NLA];   // list cursors (advance)
             uint32_t ln[NLA];          // remaining lengths (| kBmFlag: bitmap row)
@@ -368,13 +431,14 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                 ilo = (uint32_t)((o0 > t0 ? o0 : t0) - o0);
                 ihi = (uint32_t)((o1 < t1 ? o1 : t1) - o0);
                 so = src_off[e];
+                if (M == kWrite && ord_pos) obase = ord_pos[e] - ord_pos[ord_ea];
 #pragma unroll
                 for (int p = 0; p < J; ++p) path[p] = path_s[(size_t)p * W + e];
 #pragma unroll
                 for (int x = 0; x < NL; ++x) {
                     const uint64_t off = lst_off[(size_t)x * W + e];
                     ln[x] = lst_len[(size_t)x * W + e];
-                    lb[x] = ((ln[x] & kBmFlag) ? g.bm : g.col) + off;
+                    lb[x] = ((ln[x] & kBmFlag) && ln[x] != kSkip ? g.bm : g.col) + off;
                 }
             } else {
 #pragma unroll
@@ -382,8 +446,18 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
 #pragma unroll
                 for (int x = 0; x < NLA; ++x) { ln[x] = 0; lb[x] = g.col; }
             }
-            const uint32_t* __restrict__ src = g.col + so;
+            // candidate source: a CSR list (u32 stride) or an ancestor's children range
+            // in the trie (uint2 stride, .x = vertex)
+            const bool tsrc = (so & kTrieSrc) != 0;
+            // packed CSR source (degree in the id word) only where a degree filter applies
+            const bool pk = !tsrc && g.colx != nullptr && qd > 1;
+            const uint32_t* __restrict__ src = tsrc ? (const uint32_t*)(rsrc + (so & ~kTrieSrc)) : (pk ? g.colx : g.col) + so;
+            const uint32_t ssh = tsrc ? 1u : 0u;
+            const uint32_t umask = pk ? kPackMask : 0xffffffffu;
+            // an ancestor range already passed deg >= qdeg[a]: no check needed when qdeg[J] <= qdeg[a]
+            const bool dload = qd > 1 && !pk && !(tsrc && qd <= qda);
             const uint32_t nit = (ihi - ilo + G - 1) / G;
+            unsigned long long ecnt = 0, run = 0;   // per-entry count (pass A) / ordered-write cursor
             uint32_t nit_max = nit;
             if (VPW > 1) {
 #pragma unroll
@@ -393,6 +467,13 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
             auto emit = [&](bool ok, uint32_t c) {
                 if (M == kCount) {
                     my_count += ok ? 1 : 0;
+                    ecnt += ok ? 1 : 0;
+                } else if (M == kWrite && ord_pos) {
+                    // ordered write: the entry's children are contiguous at its exact offset
+                    const unsigned seg = (__ballot_sync(0xffffffffu, ok) >> vb) & kGMask;
+                    const unsigned long long pos = obase + run + __popc(seg & ((1u << vl) - 1u));
+                    run += __popc(seg);
+                    if (ok && pos < cap) out_level[pos] = make_uint2(c, (uint32_t)(w0 + e));
                 } else {
                     const unsigned m = __ballot_sync(0xffffffffu, ok);
                     const int nsel = __popc(m);
@@ -420,14 +501,15 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                 for (uint32_t it = 0; it < nit_max; it += 2) {
                     const uint32_t i0 = ilo + it * G + vl, i1 = i0 + G;
                     const bool a0 = i0 < ihi, a1 = i1 < ihi;
-                    const uint32_t c0 = a0 ? __ldg(src + i0) : 0u;
-                    const uint32_t c1 = a1 ? __ldg(src + i1) : 0u;
+                    const uint32_t r0 = a0 ? __ldg(src + ((size_t)i0 << ssh)) : 0u;
+                    const uint32_t r1 = a1 ? __ldg(src + ((size_t)i1 << ssh)) : 0u;
+                    const uint32_t c0 = r0 & umask, c1 = r1 & umask;
                     bool k0 = a0, k1 = a1;
 #pragma unroll
                     for (int p = 0; p < J; ++p) { k0 = k0 && (path[p] != c0); k1 = k1 && (path[p] != c1); }
                     if (qd > 1) {
-                        const uint32_t d0 = k0 ? __ldg(g.deg + c0) : 0u;
-                        const uint32_t d1 = k1 ? __ldg(g.deg + c1) : 0u;
+                        const uint32_t d0 = pk ? (r0 >> kPackShift) : ((k0 && dload) ? __ldg(g.deg + c0) : 0xffffffffu);
+                        const uint32_t d1 = pk ? (r1 >> kPackShift) : ((k1 && dload) ? __ldg(g.deg + c1) : 0xffffffffu);
                         k0 = k0 && d0 >= qd;
                         k1 = k1 && d1 >= qd;
                     }
@@ -440,17 +522,18 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
             for (uint32_t it = 0; it < nit_max; ++it) {
                 const uint32_t i = ilo + it * G + vl;
                 const bool act = i < ihi;
-                const uint32_t c = act ? __ldg(src + i) : 0u;
+                const uint32_t raw = act ? __ldg(src + ((size_t)i << ssh)) : 0u;
+                const uint32_t c = raw & umask;
                 bool inj = act;
 #pragma unroll
                 for (int p = 0; p < J; ++p) inj = inj && (path[p] != c);      // injectivity
                 // independent loads issued together: degree (Def. 5) and every hub-bitmap probe
                 const bool pre = count_bytes ? act : inj;
-                const uint32_t dg = (inj && qd > 1) ? __ldg(g.deg + c) : 0xffffffffu;
+                const uint32_t dg = pk ? (raw >> kPackShift) : ((inj && dload) ? __ldg(g.deg + c) : 0xffffffffu);
                 uint32_t bmw[NLA];
 #pragma unroll
                 for (int x = 0; x < NL; ++x)
-                    bmw[x] = (pre && (ln[x] & kBmFlag)) ? __ldg(lb[x] + (c >> 5)) : 0xffffffffu;
+                    bmw[x] = (pre && (ln[x] & kBmFlag) && ln[x] != kSkip) ? __ldg(lb[x] + (c >> 5)) : 0xffffffffu;
                 bool ok = inj && dg >= qd;                                    // every neighbour has deg >= 1
                 bool inter = count_bytes ? act : ok;
 #pragma unroll
@@ -486,9 +569,14 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                 emit(ok, c);
             }
             }
+            if (M == kCount && ord_cnt) {     // pass A of an ordered level: children per entry
+#pragma unroll
+                for (int o = G / 2; o >= 1; o >>= 1) ecnt += __shfl_xor_sync(0xffffffffu, ecnt, o);
+                if (has && vl == 0) ord_cnt[e] = ecnt;
+            }
         }
     }
-    if (M == kCount) {
+    if (M == kCount && !ord_cnt) {
         my_count = warp_sum(my_count);
         if (lane == 0) add_u128(ctrl + kCountLo, my_count);
     }
@@ -496,6 +584,25 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
         bytes = warp_sum(bytes);
         if (lane == 0) atomicAdd(ctrl + kBytesExt, bytes);
     }
+}
+
+// ------------------------------------------------- ordered-level chunking
+// Largest eb in [ea, W] with cpos[eb] - cpos[ea] <= cap (children of entries
+// [ea, eb) fit the level chunk).  out: eb, children, items [offs[ea], offs[eb]),
+// and for a single oversized entry its item end offs[ea+1].
+__global__ void k_find_chunk(const uint64_t* __restrict__ cpos, const uint64_t* __restrict__ offs, uint32_t W,
+                             uint32_t ea, uint64_t cap, unsigned long long* __restrict__ out) {
+    const uint64_t c0 = cpos[ea];
+    uint32_t lo = ea, hi = W;            // invariant: cpos[lo] - c0 <= cap
+    while (lo < hi) {
+        const uint32_t mid = lo + (hi - lo + 1) / 2;
+        if (cpos[mid] - c0 <= cap) lo = mid; else hi = mid - 1;
+    }
+    out[0] = lo;
+    out[1] = cpos[lo] - c0;
+    out[2] = offs[ea];
+    out[3] = offs[lo];
+    out[4] = offs[ea + 1 <= W ? ea + 1 : W];
 }
 
 // ---------------------------------------------------------- work donation

@@ -76,10 +76,12 @@ C3 = Workload(
     ((C3_GRAPH, tuple(dense_family(6) + dense_family(7) + dense_family(8))),))
 
 # configs[3]: 8-vertex dense query on R-MAT scale 22 forcing hybrid BFS/DFS chunking
-# beyond 180 GB.  R-MAT(22, 16, .50, .20, .20): K8's deepest stored level holds
-# ~5.5e11 entries over all roots (4.4 TB of trie) and the full query ~3 h on one
-# GPU; restricted to the first 1/16 of the canonical level-1 list (stated, as
-# SURVEY §8.d allows) the deepest level is still ~3.5e10 entries = 280 GB > 180 GB.
+# beyond 180 GB.  R-MAT(22, 16, .50, .20, .20), K8, restricted to the first 1/16 of
+# the canonical level-1 list (stated, as SURVEY §8.d allows).  Measured
+# (profiles/r01_c4_run_reuse.json): levels 1.1e5 / 7.8e6 / 3.3e7 / 4.0e8 / 7.6e9 /
+# 1.6e11 / 3.5e12, count 7.33e13 — the deepest stored level alone would be 28 TB of
+# 8 B trie entries (BFS stops with CUTS_ENOMEM at level 5), HYBRID finishes in
+# 1,604 s on one B200.
 C4_GRAPH = GraphSpec("rmat_t", (22, 16, 0.50, 0.20, 0.20, 1))
 C4 = Workload(
     "C4", "K8 on R-MAT(22,16,.50,.20,.20), canonical roots [0, 1/16); hybrid count beyond 180 GB",
