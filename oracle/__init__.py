@@ -95,12 +95,91 @@ def order(q) -> list:
     return out.tolist()
 
 
+# ------------------------------------------------------ disconnected queries
+# PAPER.md:544-551 (§4): "If the query graph is not connected ... we split Q
+# into a set of connected components, compute sub-graph isomorphism on each of
+# these components, and produce the final result as the cross product of
+# individual solutions."  Reading P16: an element of the result
+# is still a subgraph isomorphism (Def. 4), i.e. injective, so the
+# cross product keeps only the combinations whose images are disjoint.
+
+def components(q) -> list:
+    """Connected components of Q as sorted vertex lists, ordered by min vertex."""
+    adj = [set() for _ in range(q.k)]
+    for u, v in q.edges:
+        adj[u].add(v)
+        adj[v].add(u)
+    seen, comps = set(), []
+    for s in range(q.k):
+        if s in seen:
+            continue
+        stack, comp = [s], set()
+        while stack:
+            x = stack.pop()
+            if x in comp:
+                continue
+            comp.add(x)
+            stack.extend(adj[x] - comp)
+        seen |= comp
+        comps.append(sorted(comp))
+    return comps
+
+
+def _sub_query(q, comp):
+    """The component as its own query on vertices 0..|comp|-1 (same vertex order)."""
+    idx = {v: i for i, v in enumerate(comp)}
+    return _SubQuery(len(comp), [(idx[u], idx[v]) for u, v in q.edges if u in idx])
+
+
+class _SubQuery:
+    def __init__(self, k, edges):
+        self.k, self.edges = k, edges
+
+    def csr(self):
+        adj = [sorted({v for a, v in self.edges if a == u} | {a for a, v in self.edges if v == u})
+               for u in range(self.k)]
+        row = np.zeros(self.k + 1, dtype=np.uint32)
+        row[1:] = np.cumsum([len(a) for a in adj])
+        return row, np.asarray([v for a in adj for v in a], dtype=np.uint32)
+
+
+def _cross_product_rows(g, q) -> np.ndarray:
+    """P:546-551 step by step: per-component embeddings (the connected oracle
+    below), then their cross product, keeping injective combinations only."""
+    comps = components(q)
+    rows = np.zeros((1, q.k), dtype=np.uint32)      # the empty partial map
+    placed = []
+    for comp in comps:
+        sub = enumerate_rows(g, _sub_query(q, comp))
+        if rows.shape[0] == 0 or sub.shape[0] == 0:
+            return np.zeros((0, q.k), dtype=np.uint32)
+        a = np.repeat(rows, sub.shape[0], axis=0)
+        b = np.tile(sub, (rows.shape[0], 1))
+        ok = np.ones(a.shape[0], dtype=bool)
+        for x in placed:                              # injectivity across components
+            for y in range(len(comp)):
+                ok &= a[:, x] != b[:, y]
+        a = a[ok]
+        a[:, comp] = b[ok]
+        rows = a
+        placed.extend(comp)
+    order_ = np.lexsort(rows.T[::-1])
+    return rows[order_]
+
+
 def count(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 - 1, levels: bool = False):
     """Exact number of ordered non-induced embeddings (Python int, 128-bit).
+
+    A disconnected Q goes through the per-component cross product of P:546-551
+    (``_cross_product_rows``; no order, root range or level sizes there).
 
     With ``levels=True`` returns ``(count, [|L_0|, |L_1|, ..., |L_k|])`` where
     |L_j| counts partial paths of j matched vertices (|L_0| is 0).
     """
+    if len(components(q)) > 1:
+        if order is not None or root_begin != 0 or root_end != 2**64 - 1 or levels:
+            raise OracleError(ORC_EUNSUPPORTED)
+        return int(_cross_product_rows(g, q).shape[0])
     rp, col = _graph_arrays(g)
     qr, qc, o = _query_arrays(q, order)
     lo = np.zeros(1, np.uint64)
@@ -122,6 +201,11 @@ def count(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 - 1, leve
 def enumerate_rows(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 - 1,
                    cap_rows: int | None = None) -> np.ndarray:
     """All embeddings as a sorted (count, k) uint32 array, row[q] = f(q)."""
+    if len(components(q)) > 1:
+        if order is not None or root_begin != 0 or root_end != 2**64 - 1:
+            raise OracleError(ORC_EUNSUPPORTED)
+        rows = _cross_product_rows(g, q)
+        return rows if cap_rows is None else rows[:cap_rows]
     if cap_rows is None:
         cap_rows = count(g, q, order, root_begin, root_end)
     rp, col = _graph_arrays(g)

@@ -273,8 +273,6 @@ def test_validation():
     for g in (bad_asym, bad_loop, bad_sort):
         assert not oracle.validate_graph(g)
     with pytest.raises(oracle.OracleError):
-        oracle.count(er_graph(20, 30, 1), query_from_edges(4, [(0, 1), (2, 3)]))   # disconnected Q
-    with pytest.raises(oracle.OracleError):
         oracle.count(er_graph(20, 30, 1), named_query("P4"), order=[0, 2, 1, 3])   # order not connected
 
 
@@ -308,3 +306,51 @@ def test_rmat_torch_generator_is_byte_identical():
     for args in [(10, 8, 0.57, 0.19, 0.19, 3), (11, 16, 0.45, 0.22, 0.22, 1), (9, 4, 0.35, 0.22, 0.22, 7)]:
         a, b = rmat_graph(*args), rmat_graph_torch(*args, block=1 << 12)
         assert np.array_equal(a.row_ptr, b.row_ptr) and np.array_equal(a.col, b.col), args
+
+
+# ------------------------------------------------- disconnected Q
+# The oracle composes per-component results by the paper's cross product; these
+# pins fix it against the plain definition (injective maps) independently.
+DISCONNECTED = {
+    "2K1": (2, []), "3K1": (3, []), "K2uK1": (3, [(0, 1)]), "2K2": (4, [(0, 1), (2, 3)]),
+    "K3uK1": (4, [(0, 1), (1, 2), (0, 2)]), "P3uK2": (5, [(0, 1), (1, 2), (3, 4)]),
+    "K4uK1": (5, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)]),   # the P:1325-1327 tie member
+    "K2uK1_mid": (3, [(0, 2)]), "K3uK2": (5, [(0, 3), (3, 4), (0, 4), (1, 2)]),
+}
+
+
+@pytest.mark.parametrize("name", sorted(DISCONNECTED))
+@pytest.mark.parametrize("gi", [0, 1, 2])
+def test_disconnected_bruteforce(name, gi):
+    """Cross product of the component results, injective combinations only
+    (reading P16) == brute force over every injective vertex map."""
+    k, es = DISCONNECTED[name]
+    q = query_from_edges(k, es)
+    g = [er_graph(8, 12, 5), petersen_graph(), graph_from_edges(7, [(0, 1), (1, 2), (2, 0), (3, 4), (5, 6), (4, 5)])][gi]
+    want = bruteforce.embeddings(g, q)
+    got = [tuple(r) for r in oracle.enumerate_rows(g, q).tolist()]
+    assert got == want
+    assert oracle.count(g, q) == len(want)
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_disconnected_closed_forms(seed):
+    """kK1: falling(n, k); Q ∪ K1: count(Q) * (n - |Q|) (the isolated query
+    vertex takes any unused data vertex); 2K2: 4m^2 - 4 Σ d(v)^2 + 4m
+    (ordered edge pairs minus those sharing an endpoint)."""
+    g = er_graph(60, 150, seed)
+    d = [int(x) for x in g.degrees()]
+    m = sum(d) // 2
+    for k in (1, 2, 3):
+        assert oracle.count(g, query_from_edges(k, [])) == falling(g.n, k)
+    for qname in ("K3", "P3", "C4"):
+        q = named_query(qname)
+        qq = query_from_edges(q.k + 1, q.edges)
+        assert oracle.count(g, qq) == oracle.count(g, q) * (g.n - q.k)
+    assert oracle.count(g, query_from_edges(4, [(0, 1), (2, 3)])) == 4 * m * m - 4 * sum(x * x for x in d) + 4 * m
+
+
+def test_disconnected_complete_host():
+    """In K_n every injective map is an embedding, connected or not."""
+    for k, es in DISCONNECTED.values():
+        assert oracle.count(complete_graph(7), query_from_edges(k, es)) == math.perm(7, k)
