@@ -4,7 +4,7 @@
  * Sukumaran-Rajam, SC '21).  "P:n" cites /root/reference/PAPER.md line n.
  *
  * The library counts or enumerates the ORDERED, NON-INDUCED embeddings of a
- * small connected query graph Q (k <= 8 vertices) in a large undirected data
+ * small query graph Q (k <= 8 vertices) in a large undirected data
  * graph D (Def. 2-4; readings P1/P2 in DESIGN.md):
  *     Emb(Q, D) = { f : V_Q -> V_D injective | {u,w} in E_Q => {f(u),f(w)} in E_D }.
  * It does so the paper's way: level-synchronous extension of partial paths
@@ -48,7 +48,7 @@ typedef enum {
     CUTS_EOVERFLOW = -4,    /* count >= 2^64 (cuts_count); full value in cuts_stats     */
     CUTS_ETRUNC = -5,       /* enumeration found more rows than cap_rows                */
     CUTS_ESTATE = -6,       /* call out of order                                        */
-    CUTS_EUNSUPPORTED = -7, /* disconnected query (NEXT-3) or k > 8          */
+    CUTS_EUNSUPPORTED = -7, /* k > 8                                                    */
     CUTS_ECOMM = -8         /* reserved for the multi-GPU layer                         */
 } cuts_status;
 
@@ -130,11 +130,17 @@ cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz,
 cuts_status cuts_set_hub_threshold(cuts_ctx* ctx, uint32_t t);
 
 /* Query Q as HOST CSR over 0..k-1 (1 <= k <= 8): row_ptr u32[k+1], col u32[...],
- * symmetric, no loops/duplicates, connected (else CUTS_EUNSUPPORTED).
+ * symmetric, no loops/duplicates.  Q may be disconnected: the result
+ * is the cross product of the components' embeddings restricted to injective
+ * combinations (reading P16), built inside the same trie — a component's first
+ * matched vertex (bw = 0) takes its candidates from {v : deg(v) >= its degree}
+ * and the injectivity filter removes the overlapping combinations.
  * order == NULL -> the paper's rule: root = max degree (ties: min id),
  * then the max-degree vertex adjacent to the matched set (ties: min
- * id, reading P6).  Else order is a permutation of 0..k-1 in which every
- * order[i], i >= 1, has a neighbour in order[0..i-1] (else CUTS_EINVAL).
+ * id, reading P6); when no unmatched vertex touches the matched set, the next
+ * component starts at its max-degree vertex (ties: min id).  Else order is a
+ * permutation of 0..k-1 in which every order[i], i >= 1, has a neighbour in
+ * order[0..i-1] or is the first of its component (else CUTS_EINVAL).
  * Resets the root range and partition to "all". */
 cuts_status cuts_set_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr,
                            const uint32_t* col, const uint32_t* order);

@@ -176,16 +176,15 @@ cuts_status plan_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row, const uin
             if (!q_adj(row, col, b, a)) return fail(ctx, CUTS_EINVAL, "query not symmetric at (%u,%u)", a, b);
         }
     }
-    uint32_t seen = 1u;   // connectivity (disconnected Q is NEXT-3)
-    for (bool grown = true; grown;) {
-        grown = false;
+    // connected components: comp[a] = smallest vertex of a's component
+    uint32_t comp[CUTS_MAX_K];
+    for (uint32_t a = 0; a < k; ++a) comp[a] = a;
+    for (bool changed = true; changed;) {
+        changed = false;
         for (uint32_t a = 0; a < k; ++a)
-            if (seen >> a & 1u)
-                for (uint32_t p = row[a]; p < row[a + 1]; ++p)
-                    if (!(seen >> col[p] & 1u)) { seen |= 1u << col[p]; grown = true; }
+            for (uint32_t p = row[a]; p < row[a + 1]; ++p)
+                if (comp[col[p]] < comp[a]) { comp[a] = comp[col[p]]; changed = true; }
     }
-    if (seen != (1u << k) - 1u) return fail(ctx, CUTS_EUNSUPPORTED, "disconnected query graph (P:544-551) is not supported");
-
     uint32_t S[CUTS_MAX_K];
     auto qdeg = [&](uint32_t a) { return row[a + 1] - row[a]; };
     if (order) {
@@ -197,16 +196,20 @@ cuts_status plan_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row, const uin
         }
     } else {
         // root: max degree, ties -> min id; then max degree adjacent
-        // to the matched set, ties -> min id (reading P6)
+        // to the matched set, ties -> min id (reading P6).  When no
+        // unmatched vertex touches the matched set, the next component starts
+        // at its max-degree vertex (components in turn, reading P16)
         uint32_t used = 0;
         for (uint32_t i = 0; i < k; ++i) {
             int pick = -1;
-            for (uint32_t a = 0; a < k; ++a) {
-                if (used >> a & 1u) continue;
-                bool touches = (i == 0);
-                for (uint32_t j = 0; j < i && !touches; ++j) touches = q_adj(row, col, a, S[j]);
-                if (!touches) continue;
-                if (pick < 0 || qdeg(a) > qdeg((uint32_t)pick)) pick = (int)a;
+            for (int pass = 0; pass < 2 && pick < 0; ++pass) {
+                for (uint32_t a = 0; a < k; ++a) {
+                    if (used >> a & 1u) continue;
+                    bool touches = (i == 0) || pass == 1;
+                    for (uint32_t j = 0; j < i && !touches; ++j) touches = q_adj(row, col, a, S[j]);
+                    if (!touches) continue;
+                    if (pick < 0 || qdeg(a) > qdeg((uint32_t)pick)) pick = (int)a;
+                }
             }
             S[i] = (uint32_t)pick;
             used |= 1u << pick;
@@ -220,7 +223,9 @@ cuts_status plan_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row, const uin
         qp.bw[i] = 0;
         for (uint32_t j = 0; j < i; ++j)
             if (q_adj(row, col, S[j], S[i])) qp.bw[i] |= 1u << j;
-        if (i > 0 && qp.bw[i] == 0)
+        bool starts = true;   // no earlier position in S[i]'s component
+        for (uint32_t j = 0; j < i; ++j) starts = starts && comp[S[j]] != comp[S[i]];
+        if (i > 0 && qp.bw[i] == 0 && !starts)
             return fail(ctx, CUTS_EINVAL, "order position %u (query vertex %u) has no backward neighbour", i, S[i]);
     }
     *out = qp;
@@ -302,7 +307,7 @@ void launch_extend_nl(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t
 template <int J, int M>
 void launch_extend_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
-    const int nl = __builtin_popcount(ctx->q.bw[J]) - 1;
+    const int nl = std::max(__builtin_popcount(ctx->q.bw[J]) - 1, 0);   // component root: 0
     switch (nl) {
         case 0: launch_extend_nl<J, 0, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
         case 1: if constexpr (J > 1) launch_extend_nl<J, (J > 1 ? 1 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
@@ -765,6 +770,36 @@ cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
     return CUTS_OK;
 }
 
+// component roots (bw[J] == 0, J > 0): their candidate set is the
+// cross-product factor {v : deg(v) >= qdeg[J]}, ascending, built once per run
+// on the bottom stack (the extend kernel reads it like a CSR source list)
+cuts_status build_free_lists(cuts_ctx* ctx, Run& r) {
+    r.g.fre = (const uint32_t*)ctx->arena;
+    for (uint32_t J = 1; J < ctx->q.k; ++J) {
+        ctx->q.foff[J] = 0;
+        ctx->q.flen[J] = 0;
+        if (ctx->q.bw[J]) continue;
+        uint64_t off_list;
+        TRY(alloc_bot(ctx, (uint64_t)ctx->n * 4 + 4, &off_list));
+        const uint64_t top_save = ctx->top;
+        DegAtLeast pred{ctx->deg, ctx->q.qdeg[J]};
+        thrust::counting_iterator<uint32_t> it(0);
+        size_t tmp_bytes = 0;
+        uint64_t off_tmp;
+        uint32_t* list = (uint32_t*)(ctx->arena + off_list);
+        CK(cub::DeviceSelect::If(nullptr, tmp_bytes, it, list, ctx->ctrl + kNumSel, (int64_t)ctx->n, pred, ctx->stream));
+        TRY(alloc_top(ctx, tmp_bytes, &off_tmp));
+        CK(cub::DeviceSelect::If(ctx->arena + off_tmp, tmp_bytes, it, list, ctx->ctrl + kNumSel, (int64_t)ctx->n, pred,
+                                 ctx->stream));
+        TRY(read_ctrl(ctx));
+        ctx->top = top_save;
+        ctx->q.foff[J] = off_list / 4;
+        ctx->q.flen[J] = (uint32_t)ctx->h_ctrl[kNumSel];
+        ctx->st.launches += 2;
+    }
+    return CUTS_OK;
+}
+
 // flat-prefix seeding: levels 1..pre_j as a chain trie over the caller's rows
 cuts_status build_prefix_levels(cuts_ctx* ctx, Run& r) {
     const uint32_t J = ctx->pre_j;
@@ -808,6 +843,7 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     r.rows = rows;
     r.cap_rows = cap_rows;
     r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words, ctx->colx};
+    TRY(build_free_lists(ctx, r));
     uint64_t n1 = 0;
     const int k = (int)ctx->q.k;
     for (int j = 0; j <= kMaxK; ++j) { ctx->dfs_on[j] = false; ctx->dfs_next[j] = ctx->dfs_end[j] = 0; ctx->ord[j].valid = false; }

@@ -28,6 +28,11 @@ struct QPlan {                 // query in matching-order positions
     uint32_t S[kMaxK];         // S[i] = query vertex matched at position i
     uint32_t qdeg[kMaxK];      // deg_Q(S[i])       (degree filter)
     uint32_t bw[kMaxK];        // bit p set <=> (S[p], S[i]) in E_Q, p < i (next_neigh)
+    // bw[i] == 0, i > 0: S[i] starts another connected component of Q.
+    // Its candidates are the cross product's factor {v : deg(v) >= qdeg[i]}, a
+    // sorted list at Graph::fre + foff[i] of flen[i] entries (built per run).
+    uint64_t foff[kMaxK];
+    uint32_t flen[kMaxK];
 };
 
 struct Trie {                  // lv[l] = level l (1-based): .x = data vertex, .y = parent index in level l-1
@@ -51,6 +56,7 @@ struct Reuse {
 };
 
 constexpr uint64_t kTrieSrc = 1ull << 63;   // src_off flag: the source is a trie range
+constexpr uint64_t kFreeSrc = 1ull << 62;   // src_off flag: the source is a component's free list
 constexpr uint32_t kSkip = 0xffffffffu;     // list-slot length: no list in this slot
 
 struct Graph {
@@ -62,6 +68,7 @@ struct Graph {
     uint32_t n;
     uint32_t words;
     const uint32_t* __restrict__ colx;  // col with min(deg, 31) packed in bits 27..31 (nullptr: n >= 2^27)
+    const uint32_t* __restrict__ fre = nullptr;   // free lists of component roots (QPlan::foff/flen)
 };
 
 constexpr uint32_t kNoHub = 0xffffffffu;
@@ -294,7 +301,11 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                 if (((bw & ~ru.bwa) >> p) & 1u) { rest_min = min(rest_min, ln_[p]); rest_sum += ln_[p]; }
             if (trie_len <= rest_min) { trie = true; keep = bw & ~ru.bwa; }
         }
-        if (trie) {
+        if (bw == 0) {           // component root: cross-product factor
+            src_off[e] = q.foff[J] | kFreeSrc;
+            ub[e] = q.flen[J];
+            lists = q.flen[J];
+        } else if (trie) {
             src_off[e] = trie_off | kTrieSrc;
             ub[e] = trie_len;
             best = -1;
@@ -321,7 +332,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                     const uint32_t tl = ln_[y]; ln_[y] = ln_[y + 1]; ln_[y + 1] = tl;
                     const uint64_t tb = lb_[y]; lb_[y] = lb_[y + 1]; lb_[y + 1] = tb;
                 }
-        const int nl = __popc(bw) - 1;
+        const int nl = __popc(bw) - 1;   // -1 for a component root: no lists
 #pragma unroll
         for (int y = 0; y < J - 1; ++y)
             if (y < nl) {
@@ -449,13 +460,16 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
             // candidate source: a CSR list (u32 stride) or an ancestor's children range
             // in the trie (uint2 stride, .x = vertex)
             const bool tsrc = (so & kTrieSrc) != 0;
+            // a component root's free list is already degree-filtered
+            const bool fsrc = (so & kFreeSrc) != 0;
             // packed CSR source (degree in the id word) only where a degree filter applies
-            const bool pk = !tsrc && g.colx != nullptr && qd > 1;
-            const uint32_t* __restrict__ src = tsrc ? (const uint32_t*)(rsrc + (so & ~kTrieSrc)) : (pk ? g.colx : g.col) + so;
+            const bool pk = !tsrc && !fsrc && g.colx != nullptr && qd > 1;
+            const uint32_t* __restrict__ src = tsrc ? (const uint32_t*)(rsrc + (so & ~kTrieSrc))
+                                             : fsrc ? g.fre + (so & ~kFreeSrc) : (pk ? g.colx : g.col) + so;
             const uint32_t ssh = tsrc ? 1u : 0u;
             const uint32_t umask = pk ? kPackMask : 0xffffffffu;
             // an ancestor range already passed deg >= qdeg[a]: no check needed when qdeg[J] <= qdeg[a]
-            const bool dload = qd > 1 && !pk && !(tsrc && qd <= qda);
+            const bool dload = qd > 1 && !pk && !fsrc && !(tsrc && qd <= qda);
             const uint32_t nit = (ihi - ilo + G - 1) / G;
             unsigned long long ecnt = 0, run = 0;   // per-entry count (pass A) / ordered-write cursor
             uint32_t nit_max = nit;

@@ -282,9 +282,9 @@ def test_edge_cases(ctx):
     _set(ctx, named_query("K3"))
     rows = ctx.enumerate("bfs", cap_rows=10)
     assert ctx.truncated and rows.shape[0] == 10 and ctx.stats()["count"] == 120
-    # disconnected query / bad order / bad graph
+    # k > 8 / bad order / bad graph
     with pytest.raises(CutsError) as ei:
-        ctx.set_query_edges(4, [(0, 1), (2, 3)])
+        ctx.set_query_edges(9, [(i, i + 1) for i in range(8)])
     assert ei.value.status == -7
     with pytest.raises(CutsError) as ei:
         qr, qc = named_query("P4").csr()
@@ -350,3 +350,79 @@ def test_hub_bitmaps_parity(cuts, t):
     c.load_csr(g)
     for q in DENSE5[::3]:
         _check_full(c, g, q, modes=("hybrid",))
+
+
+# --------------------------------------------- disconnected Q (NEXT-3)
+DISCONNECTED = {
+    "2K1": (2, []), "3K1": (3, []), "K2uK1": (3, [(0, 1)]), "2K2": (4, [(0, 1), (2, 3)]),
+    "K3uK1": (4, [(0, 1), (1, 2), (0, 2)]), "P3uK2": (5, [(0, 1), (1, 2), (3, 4)]),
+    "K4uK1": (5, [(0, 1), (0, 2), (0, 3), (1, 2), (1, 3), (2, 3)]),   # the P:1325-1327 tie member
+    "K2uK1_mid": (3, [(0, 2)]), "K3uK2": (5, [(0, 3), (3, 4), (0, 4), (1, 2)]),
+    "C4uK3": (7, [(0, 1), (1, 2), (2, 3), (0, 3), (4, 5), (5, 6), (4, 6)]),
+    "K3u2K1": (5, [(0, 1), (1, 2), (0, 2)]),
+}
+
+
+@pytest.mark.parametrize("gname", ["er60", "petersen", "rmat8", "k7"])
+def test_disconnected_queries(cuts, gname):
+    """In-trie cross product (a component root extends from the degree-filtered
+    vertex list, injectivity against the path) == the oracle's per-component
+    cross product; counts in both modes, sorted rows, and a 64 KiB arena."""
+    from inputs import petersen_graph
+    g = {"er60": lambda: er_graph(60, 150, 3), "petersen": petersen_graph,
+         "rmat8": lambda: rmat_graph(8, 4, seed=2), "k7": lambda: complete_graph(7)}[gname]()
+    big = cuts(device=0, arena_bytes=1 << 28)
+    small = cuts(device=0, arena_bytes=64 << 10)
+    big.load_csr(g, validate=True)
+    small.load_csr(g)
+    for name, (k, es) in DISCONNECTED.items():
+        q = query_from_edges(k, es, name)
+        want = oracle.count(g, q)
+        _set(big, q)
+        _set(small, q)
+        assert big.count("bfs") == want, (gname, name)
+        assert big.count("hybrid") == want, (gname, name)
+        assert small.count("hybrid") == want, (gname, name)
+        if want <= 2_000_000:
+            rows = big.enumerate("hybrid", cap_rows=want)
+            assert np.array_equal(_sorted_rows(rows), oracle.enumerate_rows(g, q)), (gname, name)
+
+
+def test_disconnected_levels_and_orders(ctx):
+    """Per-level trie sizes against brute force for the order the library picks
+    and for explicit orders (components in either sequence); an order that
+    leaves a component before its root is matched is rejected."""
+    from tests import bruteforce
+    from paper_conf_sc_xiangkshs21_b200 import CutsError
+    g = er_graph(9, 16, 4)
+    ctx.load_csr(g)
+    for name, order in (("2K2", None), ("2K2", [2, 3, 0, 1]), ("P3uK2", None), ("P3uK2", [3, 4, 1, 0, 2]),
+                        ("K3uK1", [3, 0, 1, 2]), ("K3u2K1", None)):
+        k, es = DISCONNECTED[name]
+        q = query_from_edges(k, es, name)
+        _set(ctx, q, order)
+        got = ctx.count("bfs")
+        st = ctx.stats()
+        assert got == len(bruteforce.embeddings(g, q)) == oracle.count(g, q)
+        assert st["level_size"] == bruteforce.level_sizes(g, q, st["order"]), (name, order)
+        if order is not None:
+            assert st["order"] == order
+    with pytest.raises(CutsError) as ei:
+        qr, qc = query_from_edges(5, DISCONNECTED["P3uK2"][1]).csr()
+        ctx.set_query(qr, qc, [0, 3, 2, 4, 1])   # vertex 2 has no backward neighbour, 0 already placed
+    assert ei.value.status == -1
+
+
+def test_disconnected_fullsize_closed_forms(cuts):
+    """At the C2 bench graph's full size (R-MAT(16,16,.45,.22,.22)): Q ∪ K1 =
+    count(Q) * (n - |Q|) for the oracle-counted K3; 2K2 = 4m^2 - 4 Σ d^2 + 4m."""
+    g = rmat_graph(16, 16, 0.45, 0.22, 0.22, seed=1)
+    c = cuts(device=0)
+    c.load_csr(g)
+    d = np.diff(g.row_ptr.astype(np.int64))
+    m = int(d.sum()) // 2
+    k3 = oracle.count(g, named_query("K3"))
+    c.set_query_edges(4, [(0, 1), (1, 2), (0, 2)])
+    assert c.count("hybrid") == k3 * (g.n - 3)
+    c.set_query_edges(4, [(0, 1), (2, 3)])
+    assert c.count("hybrid") == 4 * m * m - 4 * int((d * d).sum()) + 4 * m
