@@ -10,6 +10,9 @@ from .graphs import (CSRGraph, canonical_csr, er_graph, rmat_graph, rmat_graph_t
                      complete_graph, path_graph, star_graph, grid_graph,
                      petersen_graph, hypercube_graph, complete_bipartite_graph,
                      graph_from_edges)
+from .digraphs import (DiGraph, DiQuery, digraph_from_arcs, directed_er_graph, directed_rmat_graph,
+                       directed_cycle, transitive_tournament, complete_digraph, query_from_arcs,
+                       named_diquery, DIRECTED_QUERIES)
 from .queries import (Query, query_from_edges, k_minus, DENSE5, SPARSE5, m11,
                       dense_family, named_query)
 
@@ -19,4 +22,7 @@ __all__ = [
     "hypercube_graph", "complete_bipartite_graph", "graph_from_edges",
     "Query", "query_from_edges", "k_minus", "DENSE5", "SPARSE5", "m11",
     "dense_family", "named_query",
+    "DiGraph", "DiQuery", "digraph_from_arcs", "directed_er_graph", "directed_rmat_graph",
+    "directed_cycle", "transitive_tournament", "complete_digraph", "query_from_arcs",
+    "named_diquery", "DIRECTED_QUERIES",
 ]

@@ -50,6 +50,11 @@ def _load():
         lib.oracle_level1_size.argtypes = [ctypes.c_uint32, u64p, ctypes.c_uint32, u64p]
         lib.oracle_trie_decode.argtypes = [ctypes.c_uint32, u64p, ctypes.POINTER(u32p),
                                            ctypes.POINTER(u32p), u32p]
+        lib.oracle_di_count.argtypes = [ctypes.c_uint32, u64p, u32p, u64p, u32p, ctypes.c_uint32, u32p, u32p,
+                                        u32p, u64p, u64p, u64p, u64p, u32p, ctypes.c_uint64]
+        lib.oracle_di_order.argtypes = [ctypes.c_uint32, u32p, u32p, u32p]
+        lib.oracle_di_count.restype = ctypes.c_int
+        lib.oracle_di_order.restype = ctypes.c_int
         for f in (lib.oracle_count, lib.oracle_enumerate, lib.oracle_order,
                   lib.oracle_validate_graph, lib.oracle_level1_size, lib.oracle_trie_decode):
             f.restype = ctypes.c_int
@@ -240,3 +245,48 @@ def trie_decode(ca_levels, pa_levels) -> np.ndarray:
     out = np.zeros((int(sizes[-1]), L), dtype=np.uint32)
     _check(_load().oracle_trie_decode(L, _p(sizes, ctypes.c_uint64), ca_arr, pa_arr, _p(out, ctypes.c_uint32)))
     return out
+
+
+# ------------------------------------------------------------ directed (NEXT-1)
+def _di_call(g, q, order, rows=None, cap=0, levels=False):
+    arrs = [np.ascontiguousarray(a, dtype=t) for a, t in
+            ((g.out_row, np.uint64), (g.out_col, np.uint32), (g.in_row, np.uint64), (g.in_col, np.uint32))]
+    arrs = [a if a.size else np.zeros(1, a.dtype) for a in arrs]
+    qr, qc = q.csr()
+    qc = qc if qc.size else np.zeros(1, np.uint32)
+    qr, qc = np.ascontiguousarray(qr), np.ascontiguousarray(qc)
+    o = None if order is None else np.ascontiguousarray(order, dtype=np.uint32)
+    lo, hi = np.zeros(1, np.uint64), np.zeros(1, np.uint64)
+    llo, lhi = np.zeros(q.k + 1, np.uint64), np.zeros(q.k + 1, np.uint64)
+    _check(_load().oracle_di_count(
+        g.n, _p(arrs[0], ctypes.c_uint64), _p(arrs[1], ctypes.c_uint32), _p(arrs[2], ctypes.c_uint64),
+        _p(arrs[3], ctypes.c_uint32), q.k, _p(qr, ctypes.c_uint32), _p(qc, ctypes.c_uint32),
+        None if o is None else _p(o, ctypes.c_uint32), _p(lo, ctypes.c_uint64), _p(hi, ctypes.c_uint64),
+        _p(llo, ctypes.c_uint64), _p(lhi, ctypes.c_uint64),
+        None if rows is None else _p(rows, ctypes.c_uint32), cap))
+    total = int(lo[0]) | (int(hi[0]) << 64)
+    if levels:
+        return total, [int(a) | (int(b) << 64) for a, b in zip(llo, lhi)]
+    return total
+
+
+def di_count(g, q, order=None, levels: bool = False):
+    """Directed: exact number of injective arc-preserving maps (cuts_oracle.c
+    'directed' section: P:207-209, c-/p-intersection of Alg. 2)."""
+    return _di_call(g, q, order, levels=levels)
+
+
+def di_enumerate_rows(g, q, order=None) -> np.ndarray:
+    n = _di_call(g, q, order)
+    rows = np.zeros((max(n, 1), q.k), dtype=np.uint32)
+    _di_call(g, q, order, rows=rows, cap=n)
+    return rows[:n]
+
+
+def di_order(q) -> list:
+    qr, qc = q.csr()
+    qc = qc if qc.size else np.zeros(1, np.uint32)
+    out = np.zeros(q.k, dtype=np.uint32)
+    _check(_load().oracle_di_order(q.k, _p(np.ascontiguousarray(qr), ctypes.c_uint32),
+                                   _p(np.ascontiguousarray(qc), ctypes.c_uint32), _p(out, ctypes.c_uint32)))
+    return out.tolist()

@@ -312,3 +312,189 @@ int oracle_trie_decode(uint32_t nlevels, const uint64_t* sizes,
     }
     return ORC_OK;
 }
+
+/* ====================================================== directed (NEXT-1)
+ * "we consider directed graphs (edges are directed)"; an undirected
+ * graph is the special case with both arcs.  Plain definition (reading P1 for
+ * directed graphs):
+ *   Emb(Q, D) = { f injective | (u,w) in E_Q => (f(u),f(w)) in E_D }.
+ * The data graph is given as out-CSR (children, D.cs) and in-CSR (parents,
+ * D.ps), both sorted.  Step by step:
+ *   - order: root = max out-degree ("out degree in the case of directed
+ *     graphs"; reading P26), ties min id; next = max out-degree unmatched
+ *     vertex weakly adjacent to the matched set (P:545 weak connectivity),
+ *     ties min id.  Q must be weakly connected.
+ *   - degree filter (Def. 5, with "degree (in degree and out
+ *     degree)" of P:262-264; reading P27): outdeg(c) >= outdeg_Q(S[i]) and
+ *     indeg(c) >= indeg_Q(S[i]).
+ *   - extension of position i: for every backward neighbour j, an arc
+ *     S[j] -> S[i] requires c in children(f(S[j])) (c-intersection, Alg. 2
+ *     l.19-31) and an arc S[i] -> S[j] requires c in parents(f(S[j]))
+ *     (p-intersection, Alg. 2 l.33-42).  The initial set is the
+ *     first requirement's list (children before parents, lower j first).
+ */
+typedef struct {
+    uint32_t n;
+    const uint64_t *orow, *irow;
+    const uint32_t *ocol, *icol;
+    uint32_t k;
+    uint32_t S[ORC_MAXK];
+    uint32_t qout[ORC_MAXK], qin[ORC_MAXK];
+    uint32_t nreq[ORC_MAXK];
+    uint32_t req_pos[ORC_MAXK][2 * ORC_MAXK];   /* backward position j                    */
+    uint32_t req_par[ORC_MAXK][2 * ORC_MAXK];   /* 0: c in children(f(S[j])), 1: parents  */
+    uint32_t f[ORC_MAXK];
+    u128 level[ORC_MAXK + 1];
+    uint32_t* rows;
+    uint64_t cap_rows;
+    u128 n_rows;
+} orc_di;
+
+static int di_in_list(const uint64_t* row, const uint32_t* col, uint32_t v, uint32_t c) {
+    uint64_t b = row[v], e = row[v + 1];
+    if (e == b) return 0;
+    return bsearch(&c, col + b, (size_t)(e - b), sizeof(uint32_t), cmp_u32) != NULL;
+}
+
+static int di_q_arc(const uint32_t* qrow, const uint32_t* qcol, uint32_t a, uint32_t b) {
+    for (uint32_t p = qrow[a]; p < qrow[a + 1]; ++p)
+        if (qcol[p] == b) return 1;
+    return 0;
+}
+
+/* out-degree of query vertex a; in-degree by scanning every row */
+static uint32_t di_q_out(const uint32_t* qrow, uint32_t a) { return qrow[a + 1] - qrow[a]; }
+static uint32_t di_q_in(uint32_t k, const uint32_t* qrow, const uint32_t* qcol, uint32_t a) {
+    uint32_t c = 0;
+    for (uint32_t u = 0; u < k; ++u) c += (uint32_t)di_q_arc(qrow, qcol, u, a);
+    return c;
+}
+
+static int di_setup(orc_di* st, uint32_t n, const uint64_t* orow, const uint32_t* ocol,
+                    const uint64_t* irow, const uint32_t* icol, uint32_t k,
+                    const uint32_t* qrow, const uint32_t* qcol, const uint32_t* order) {
+    memset(st, 0, sizeof(*st));
+    st->n = n; st->orow = orow; st->ocol = ocol; st->irow = irow; st->icol = icol; st->k = k;
+    if (k < 1 || k > ORC_MAXK || qrow[0] != 0) return ORC_EINVAL;
+    for (uint32_t a = 0; a < k; ++a) {
+        if (qrow[a + 1] < qrow[a]) return ORC_EINVAL;
+        for (uint32_t p = qrow[a]; p < qrow[a + 1]; ++p) {
+            if (qcol[p] >= k || qcol[p] == a) return ORC_EINVAL;
+            for (uint32_t p2 = qrow[a]; p2 < p; ++p2)
+                if (qcol[p2] == qcol[p]) return ORC_EINVAL;
+        }
+    }
+    uint32_t used[ORC_MAXK] = {0};
+    if (order) {
+        for (uint32_t i = 0; i < k; ++i) {
+            if (order[i] >= k || used[order[i]]) return ORC_EINVAL;
+            used[order[i]] = 1;
+            st->S[i] = order[i];
+        }
+    } else {
+        for (uint32_t i = 0; i < k; ++i) {
+            int pick = -1;
+            for (uint32_t a = 0; a < k; ++a) {
+                if (used[a]) continue;
+                int touches = (i == 0);
+                for (uint32_t j = 0; j < i; ++j)
+                    if (di_q_arc(qrow, qcol, a, st->S[j]) || di_q_arc(qrow, qcol, st->S[j], a)) touches = 1;
+                if (!touches) continue;
+                if (pick < 0 || di_q_out(qrow, a) > di_q_out(qrow, (uint32_t)pick)) pick = (int)a;
+            }
+            if (pick < 0) return ORC_EUNSUPPORTED;   /* not weakly connected */
+            st->S[i] = (uint32_t)pick; used[pick] = 1;
+        }
+    }
+    for (uint32_t i = 0; i < k; ++i) {
+        uint32_t a = st->S[i];
+        st->qout[i] = di_q_out(qrow, a);
+        st->qin[i] = di_q_in(k, qrow, qcol, a);
+        for (uint32_t j = 0; j < i; ++j)
+            if (di_q_arc(qrow, qcol, st->S[j], a)) { st->req_pos[i][st->nreq[i]] = j; st->req_par[i][st->nreq[i]++] = 0; }
+        for (uint32_t j = 0; j < i; ++j)
+            if (di_q_arc(qrow, qcol, a, st->S[j])) { st->req_pos[i][st->nreq[i]] = j; st->req_par[i][st->nreq[i]++] = 1; }
+        if (i > 0 && st->nreq[i] == 0) return order ? ORC_EINVAL : ORC_EUNSUPPORTED;
+    }
+    return ORC_OK;
+}
+
+static void di_emit(orc_di* st) {
+    if (st->rows && st->n_rows < (u128)st->cap_rows) {
+        uint32_t* r = st->rows + (uint64_t)st->n_rows * st->k;
+        for (uint32_t i = 0; i < st->k; ++i) r[st->S[i]] = st->f[i];
+    }
+    st->n_rows++;
+}
+
+static int di_degree_ok(const orc_di* st, uint32_t c, uint32_t i) {
+    return st->orow[c + 1] - st->orow[c] >= st->qout[i] && st->irow[c + 1] - st->irow[c] >= st->qin[i];
+}
+
+static void di_rec(orc_di* st, uint32_t i) {
+    uint32_t v0 = st->f[st->req_pos[i][0]];
+    const uint64_t* row = st->req_par[i][0] ? st->irow : st->orow;
+    const uint32_t* col = st->req_par[i][0] ? st->icol : st->ocol;
+    for (uint64_t p = row[v0]; p < row[v0 + 1]; ++p) {
+        uint32_t c = col[p];
+        int ok = 1;
+        for (uint32_t t = 1; t < st->nreq[i] && ok; ++t) {
+            uint32_t v = st->f[st->req_pos[i][t]];
+            ok = st->req_par[i][t] ? di_in_list(st->irow, st->icol, v, c)   /* p-intersection */
+                                   : di_in_list(st->orow, st->ocol, v, c);  /* c-intersection */
+        }
+        if (!ok || !di_degree_ok(st, c, i)) continue;
+        for (uint32_t j = 0; j < i && ok; ++j) ok = st->f[j] != c;
+        if (!ok) continue;
+        st->f[i] = c;
+        st->level[i + 1]++;
+        if (i + 1 == st->k) di_emit(st);
+        else di_rec(st, i + 1);
+    }
+}
+
+static void di_run(orc_di* st) {
+    for (uint32_t v = 0; v < st->n; ++v) {
+        if (!di_degree_ok(st, v, 0)) continue;
+        st->f[0] = v;
+        st->level[1]++;
+        if (st->k == 1) di_emit(st);
+        else di_rec(st, 1);
+    }
+}
+
+/* Directed count (+ level sizes, k+1 entries, may be NULL) / enumerate. */
+int oracle_di_count(uint32_t n, const uint64_t* orow, const uint32_t* ocol, const uint64_t* irow,
+                    const uint32_t* icol, uint32_t k, const uint32_t* qrow, const uint32_t* qcol,
+                    const uint32_t* order, uint64_t* count_lo, uint64_t* count_hi,
+                    uint64_t* level_lo, uint64_t* level_hi, uint32_t* rows, uint64_t cap_rows) {
+    orc_di* st = (orc_di*)malloc(sizeof(orc_di));
+    if (!st) return ORC_ENOMEM;
+    int rc = di_setup(st, n, orow, ocol, irow, icol, k, qrow, qcol, order);
+    if (rc) { free(st); return rc; }
+    st->rows = rows; st->cap_rows = rows ? cap_rows : 0;
+    di_run(st);
+    *count_lo = (uint64_t)st->n_rows;
+    *count_hi = (uint64_t)(st->n_rows >> 64);
+    for (uint32_t j = 0; j <= k; ++j) {
+        if (level_lo) level_lo[j] = (uint64_t)st->level[j];
+        if (level_hi) level_hi[j] = (uint64_t)(st->level[j] >> 64);
+    }
+    if (rows) {
+        uint64_t nr = st->n_rows < (u128)cap_rows ? (uint64_t)st->n_rows : cap_rows;
+        g_sort_k = k;
+        qsort(rows, (size_t)nr, (size_t)k * sizeof(uint32_t), cmp_row);
+    }
+    free(st);
+    return ORC_OK;
+}
+
+int oracle_di_order(uint32_t k, const uint32_t* qrow, const uint32_t* qcol, uint32_t* order) {
+    orc_di* st = (orc_di*)malloc(sizeof(orc_di));
+    if (!st) return ORC_ENOMEM;
+    uint64_t z[2] = {0, 0};
+    int rc = di_setup(st, 0, z, NULL, z, NULL, k, qrow, qcol, NULL);
+    if (!rc) memcpy(order, st->S, k * sizeof(uint32_t));
+    free(st);
+    return rc;
+}

@@ -46,3 +46,31 @@ def level_sizes(g, q, order):
             cnt += ok
         sizes.append(cnt)
     return sizes
+
+
+# ------------------------------------------------------------------- directed
+def di_embeddings(g, q):
+    """Injective maps f with (u, v) in arcs(Q) => (f(u), f(v)) in arcs(D)."""
+    arcs = {(int(a), int(b)) for a, b in g.arcs()}
+    return sorted(f for f in permutations(range(g.n), q.k) if all((f[u], f[v]) in arcs for u, v in q.arcs))
+
+
+def di_level_sizes(g, q, order):
+    """|L_j| for the directed trie: injective maps of order[0..j-1] preserving
+    the arcs among those positions with outdeg/indeg >= the query's."""
+    arcs = {(int(a), int(b)) for a, b in g.arcs()}
+    od, idg = g.out_degrees(), g.in_degrees()
+    qo = [sum(1 for u, _ in q.arcs if u == a) for a in range(q.k)]
+    qi = [sum(1 for _, v in q.arcs if v == a) for a in range(q.k)]
+    sizes = [0]
+    for j in range(1, q.k + 1):
+        pos = order[:j]
+        ix = {p: i for i, p in enumerate(pos)}
+        inner = [(ix[u], ix[v]) for u, v in q.arcs if u in ix and v in ix]
+        cnt = 0
+        for f in permutations(range(g.n), j):
+            if any(od[f[i]] < qo[pos[i]] or idg[f[i]] < qi[pos[i]] for i in range(j)):
+                continue
+            cnt += all((f[a], f[b]) in arcs for a, b in inner)
+        sizes.append(cnt)
+    return sizes

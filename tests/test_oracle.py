@@ -354,3 +354,74 @@ def test_disconnected_complete_host():
     """In K_n every injective map is an embedding, connected or not."""
     for k, es in DISCONNECTED.values():
         assert oracle.count(complete_graph(7), query_from_edges(k, es)) == math.perm(7, k)
+
+
+# ------------------------------------------------------- directed (NEXT-1)
+from inputs import (directed_er_graph, directed_rmat_graph, directed_cycle, transitive_tournament,
+                    complete_digraph, digraph_from_arcs, query_from_arcs, named_diquery, DIRECTED_QUERIES)
+
+
+@pytest.mark.parametrize("qname", sorted(DIRECTED_QUERIES))
+def test_directed_closed_forms(qname):
+    """Complete digraph: every injective map (n!/(n-k)!).  Transitive
+    tournament: a query embeds iff it is acyclic, C(n, k) maps for TT_k."""
+    q = named_diquery(qname)
+    assert oracle.di_count(complete_digraph(7), q) == math.perm(7, q.k)
+    if qname.startswith("TT"):
+        assert oracle.di_count(transitive_tournament(8), q) == math.comb(8, q.k)
+    if qname.startswith("dC"):
+        assert oracle.di_count(transitive_tournament(8), q) == 0
+
+
+@pytest.mark.parametrize("n", [3, 4, 5, 7])
+def test_directed_cycles_and_paths(n):
+    for k in (3, 4, 5):
+        want = n if k == n else 0
+        assert oracle.di_count(directed_cycle(n), named_diquery(f"dC{k}")) == want
+    assert oracle.di_count(directed_cycle(n), named_diquery("dP3")) == n
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_directed_degree_sequence_forms(seed):
+    """out-star: Σ out(out-1); in-star: Σ in(in-1); dP3 a->b->c (a != c):
+    Σ_b in(b) out(b) - 2 * #reciprocal pairs."""
+    g = directed_er_graph(200, 1500, seed)
+    od, idg = g.out_degrees(), g.in_degrees()
+    arcs = {(int(a), int(b)) for a, b in g.arcs()}
+    recip = sum(1 for a, b in arcs if (b, a) in arcs) // 2
+    assert recip > 0
+    assert oracle.di_count(g, named_diquery("out2")) == int((od * (od - 1)).sum())
+    assert oracle.di_count(g, named_diquery("in2")) == int((idg * (idg - 1)).sum())
+    assert oracle.di_count(g, named_diquery("dP3")) == int((od * idg).sum()) - 2 * recip
+
+
+@pytest.mark.parametrize("gi", [0, 1, 2])
+def test_directed_bruteforce(gi):
+    g = [directed_er_graph(7, 18, 3), directed_er_graph(8, 25, 4), directed_rmat_graph(3, 4, seed=5)][gi]
+    for name in ("dP3", "dC3", "TT3", "out2", "in2", "dC4", "TT4", "bifan", "diamond"):
+        q = named_diquery(name)
+        want = bruteforce.di_embeddings(g, q)
+        assert [tuple(r) for r in oracle.di_enumerate_rows(g, q).tolist()] == want, name
+        c, lv = oracle.di_count(g, q, levels=True)
+        assert c == len(want)
+        assert lv == bruteforce.di_level_sizes(g, q, oracle.di_order(q)), name
+
+
+def test_directed_reduces_to_undirected():
+    """an undirected graph is the digraph with both arcs; with
+    symmetric queries (reciprocal arcs) the directed oracle equals the
+    undirected one."""
+    g = er_graph(40, 120, 7)
+    dg = digraph_from_arcs(g.n, [(int(u), int(v)) for u, v in g.edge_list()] +
+                           [(int(v), int(u)) for u, v in g.edge_list()])
+    for qname in ("K3", "C4", "P4", "K4", "S3"):
+        q = named_query(qname)
+        dq = query_from_arcs(q.k, list(q.edges) + [(v, u) for u, v in q.edges])
+        assert oracle.di_count(dg, dq) == oracle.count(g, q), qname
+
+
+def test_directed_order_rule():
+    """Root = max out-degree, ties min id; then weakly adjacent."""
+    assert oracle.di_order(named_diquery("in2")) == [1, 0, 2]
+    assert oracle.di_order(named_diquery("out2")) == [0, 1, 2]
+    assert oracle.di_order(named_diquery("TT6-rev")) == [5, 4, 3, 2, 1, 0]
