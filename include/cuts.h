@@ -121,6 +121,19 @@ int cuts_version(void);
 cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz,
                             const uint64_t* d_row_ptr, const uint32_t* d_col, int validate);
 
+/* Directed data graph ("we consider directed graphs"; NEXT-1) as ONE
+ * DEVICE CSR of 2n rows: rows 0..n-1 are the out-lists (children, the paper's
+ * D.cs), rows n..2n-1 the in-lists (parents, D.ps, used by the p-intersection
+ * of Alg. 2 l.33-42).  d_row_ptr u64[2n+1], d_col u32[nnz] with
+ * nnz = 2 x arcs; every row strictly ascending, ids < n, no loops; the in-rows
+ * must be the transpose of the out-rows (checked when validate != 0, else
+ * CUTS_EINVAL).  2n < 2^32-1.  Borrowed like cuts_load_graph's arrays.  Hub
+ * bitmaps and the packed candidate stream are not used for directed graphs.
+ * Pair with cuts_set_query_directed (an undirected query on a directed graph,
+ * or the reverse, fails at count time with CUTS_EINVAL). */
+cuts_status cuts_load_digraph(cuts_ctx* ctx, uint32_t n, uint64_t nnz,
+                              const uint64_t* d_row_ptr, const uint32_t* d_col, int validate);
+
 /* Membership rows for hub vertices (SV-style intersection, Alg. 2 l.7-17,
  * P:1055-1072): at the next cuts_load_graph, every vertex with deg >= t gets a
  * bitmap of its neighbours over [0, n) in the arena, and a membership test
@@ -144,6 +157,18 @@ cuts_status cuts_set_hub_threshold(cuts_ctx* ctx, uint32_t t);
  * Resets the root range and partition to "all". */
 cuts_status cuts_set_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr,
                            const uint32_t* col, const uint32_t* order);
+
+/* Directed query Q as HOST out-CSR over 0..k-1 (row_ptr u32[k+1], col u32:
+ * arcs a -> col[p]), no loops/duplicate arcs.  Embeddings are the injective f
+ * with (u,w) in arcs(Q) => (f(u),f(w)) in arcs(D) (reading P1, directed).
+ * Degree filter: outdeg(c) >= outdeg_Q and indeg(c) >= indeg_Q (Def. 5 with the
+ * in/out degree of P:262-264; reading P27).  order == NULL -> root = max
+ * out-degree (ties min id), then the max out-degree vertex weakly
+ * adjacent to the matched set; weak components in turn.  A position
+ * whose backward arcs need more lists than its index (reciprocal query arcs
+ * u <-> w at that position) returns CUTS_EUNSUPPORTED. */
+cuts_status cuts_set_query_directed(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr,
+                                    const uint32_t* col, const uint32_t* order);
 
 /* Restrict the roots to positions [begin, end) of the CANONICAL level-1 list
  * (vertices with deg >= deg_Q(S[0]) in ascending id, before shuffling; Alg. 1

@@ -22,6 +22,7 @@ MAX_K = 8
 
 # the symbols include/cuts.h declares (tests check the library exports all of them)
 EXPORTED = ["cuts_version", "cuts_create", "cuts_destroy", "cuts_last_error", "cuts_load_graph",
+            "cuts_load_digraph", "cuts_set_query_directed",
             "cuts_set_query", "cuts_set_root_range", "cuts_set_root_slice", "cuts_level1_size", "cuts_count",
             "cuts_enumerate", "cuts_get_stats", "cuts_set_debug", "cuts_trie_decode", "cuts_set_hub_threshold",
             "cuts_set_prefixes", "cuts_set_donation"]
@@ -70,6 +71,8 @@ def load() -> ctypes.CDLL:
         "cuts_last_error": ([P], ctypes.c_char_p),
         "cuts_load_graph": ([P, u32, u64, P, P, i32], i32),
         "cuts_set_query": ([P, u32, u32p, u32p, u32p], i32),
+        "cuts_load_digraph": ([P, u32, u64, P, P, i32], i32),
+        "cuts_set_query_directed": ([P, u32, u32p, u32p, u32p], i32),
         "cuts_set_root_range": ([P, u64, u64], i32),
         "cuts_set_root_slice": ([P, u64, u64, u32, u32], i32),
         "cuts_level1_size": ([P, u64p, u64p], i32),

@@ -90,7 +90,7 @@ class Cuts:
             pass
 
     # ------------------------------------------------------------------- API
-    def load_graph(self, row_ptr, col, validate: bool = False):
+    def load_graph(self, row_ptr, col, validate: bool = False, directed: bool = False):
         rp = torch.as_tensor(np.asarray(row_ptr, dtype=np.uint64).view(np.int64)) if not torch.is_tensor(row_ptr) else row_ptr
         cl = torch.as_tensor(np.asarray(col, dtype=np.uint32).view(np.int32)) if not torch.is_tensor(col) else col
         rp = rp.to(self.device, non_blocking=False).contiguous()
@@ -102,8 +102,12 @@ class Cuts:
             nnz = cl.numel()
         assert rp.element_size() == 8 and cl.element_size() == 4
         n = rp.numel() - 1
+        if directed:       # 2n rows: out-lists then in-lists (cuts_load_digraph)
+            assert n % 2 == 0
+            n //= 2
         self._graph = (rp, cl)   # keep the borrowed buffers alive
-        self._check(self.lib.cuts_load_graph(self.h, n, nnz, rp.data_ptr(), cl.data_ptr(), int(validate)))
+        load = self.lib.cuts_load_digraph if directed else self.lib.cuts_load_graph
+        self._check(load(self.h, n, nnz, rp.data_ptr(), cl.data_ptr(), int(validate)))
         self.n = n
         return self
 
@@ -111,7 +115,22 @@ class Cuts:
         """Load an ``inputs.CSRGraph``-like object (row_ptr, col attributes)."""
         return self.load_graph(g.row_ptr, g.col, validate)
 
-    def set_query(self, row_ptr, col, order=None):
+    def load_digraph(self, g, validate: bool = False):
+        """Load an ``inputs.DiGraph``-like object (out/in CSR) as one 2n-row CSR."""
+        rp, cl = g.combined()
+        return self.load_graph(rp, cl, validate, directed=True)
+
+    def set_query_directed(self, row_ptr, col, order=None):
+        """Directed query as out-CSR over 0..k-1 (cuts_set_query_directed)."""
+        return self.set_query(row_ptr, col, order, directed=True)
+
+    def set_query_arcs(self, k: int, arcs, order=None):
+        adj = [sorted({v for u, v in arcs if u == a}) for a in range(k)]
+        rp = np.zeros(k + 1, dtype=np.uint32)
+        rp[1:] = np.cumsum([len(x) for x in adj])
+        return self.set_query_directed(rp, np.asarray([v for x in adj for v in x], dtype=np.uint32), order)
+
+    def set_query(self, row_ptr, col, order=None, directed: bool = False):
         qr = np.ascontiguousarray(row_ptr, dtype=np.uint32)
         qc = np.ascontiguousarray(col, dtype=np.uint32)
         if qc.size == 0:
@@ -122,7 +141,8 @@ class Cuts:
         if order is not None:
             o = np.ascontiguousarray(order, dtype=np.uint32)
             op = o.ctypes.data_as(u32p)
-        self._check(self.lib.cuts_set_query(self.h, k, qr.ctypes.data_as(u32p), qc.ctypes.data_as(u32p), op))
+        fn = self.lib.cuts_set_query_directed if directed else self.lib.cuts_set_query
+        self._check(fn(self.h, k, qr.ctypes.data_as(u32p), qc.ctypes.data_as(u32p), op))
         self.k = k
         return self
 

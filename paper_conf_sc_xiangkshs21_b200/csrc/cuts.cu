@@ -49,6 +49,7 @@ struct cuts_ctx {
     unsigned long long* h_ctrl = nullptr; // pinned host mirror
     // graph
     bool has_graph = false;
+    bool directed = false;                 // cuts_load_digraph: 2n rows (out-lists, then in-lists)
     uint32_t n = 0;
     uint64_t nnz = 0;
     const uint64_t* row_ptr = nullptr;
@@ -63,6 +64,7 @@ struct cuts_ctx {
     uint64_t base_off = 0;                 // first free byte after ctrl + deg + bitmaps
     // query
     bool has_query = false;
+    bool q_directed = false;
     QPlan q{};
     uint64_t root_begin = 0, root_end = ~0ull;
     uint64_t slice_begin = 0, slice_end = ~0ull;
@@ -232,6 +234,83 @@ cuts_status plan_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row, const uin
     return CUTS_OK;
 }
 
+// ---- directed query planning (NEXT-1) ---------------------
+// Q as out-CSR over 0..k-1.  Order: root = max out-degree ("out degree in the
+// case of directed graphs"; ties min id), then the max out-degree vertex
+// weakly adjacent to the matched set, a new weak component when none is.
+// bw[i] bit p: arc S[p] -> S[i] (children list, c-intersection); bwi[i] bit p:
+// arc S[i] -> S[p] (parents list, p-intersection, Alg. 2 l.33-42).
+cuts_status plan_query_directed(cuts_ctx* ctx, uint32_t k, const uint32_t* row, const uint32_t* col,
+                                const uint32_t* order, QPlan* out) {
+    if (k < 1 || k > CUTS_MAX_K) return fail(ctx, k > CUTS_MAX_K ? CUTS_EUNSUPPORTED : CUTS_EINVAL, "k=%u out of range 1..8", k);
+    if (!row || (row[k] > 0 && !col)) return fail(ctx, CUTS_EINVAL, "null query arrays");
+    if (row[0] != 0) return fail(ctx, CUTS_EINVAL, "query row_ptr[0] != 0");
+    for (uint32_t a = 0; a < k; ++a) {
+        if (row[a + 1] < row[a]) return fail(ctx, CUTS_EINVAL, "query row_ptr not monotone");
+        for (uint32_t p = row[a]; p < row[a + 1]; ++p) {
+            if (col[p] >= k || col[p] == a) return fail(ctx, CUTS_EINVAL, "query arc (%u,%u) invalid", a, col[p]);
+            for (uint32_t p2 = row[a]; p2 < p; ++p2)
+                if (col[p2] == col[p]) return fail(ctx, CUTS_EINVAL, "duplicate query arc (%u,%u)", a, col[p]);
+        }
+    }
+    auto arc = [&](uint32_t a, uint32_t b) { return q_adj(row, col, a, b); };
+    auto weak = [&](uint32_t a, uint32_t b) { return arc(a, b) || arc(b, a); };
+    auto outd = [&](uint32_t a) { return row[a + 1] - row[a]; };
+    uint32_t comp[CUTS_MAX_K];
+    for (uint32_t a = 0; a < k; ++a) comp[a] = a;
+    for (bool changed = true; changed;) {
+        changed = false;
+        for (uint32_t a = 0; a < k; ++a)
+            for (uint32_t b = 0; b < k; ++b)
+                if (weak(a, b) && comp[b] < comp[a]) { comp[a] = comp[b]; changed = true; }
+    }
+    uint32_t S[CUTS_MAX_K];
+    uint32_t used = 0;
+    if (order) {
+        for (uint32_t i = 0; i < k; ++i) {
+            if (order[i] >= k || (used >> order[i] & 1u)) return fail(ctx, CUTS_EINVAL, "order is not a permutation");
+            used |= 1u << order[i];
+            S[i] = order[i];
+        }
+    } else {
+        for (uint32_t i = 0; i < k; ++i) {
+            int pick = -1;
+            for (int pass = 0; pass < 2 && pick < 0; ++pass)
+                for (uint32_t a = 0; a < k; ++a) {
+                    if (used >> a & 1u) continue;
+                    bool touches = (i == 0) || pass == 1;
+                    for (uint32_t j = 0; j < i && !touches; ++j) touches = weak(a, S[j]);
+                    if (!touches) continue;
+                    if (pick < 0 || outd(a) > outd((uint32_t)pick)) pick = (int)a;
+                }
+            S[i] = (uint32_t)pick;
+            used |= 1u << pick;
+        }
+    }
+    QPlan qp{};
+    qp.k = k;
+    for (uint32_t i = 0; i < k; ++i) {
+        qp.S[i] = S[i];
+        qp.qdeg[i] = outd(S[i]);
+        qp.qdin[i] = 0;
+        for (uint32_t a = 0; a < k; ++a) qp.qdin[i] += arc(a, S[i]) ? 1u : 0u;
+        for (uint32_t j = 0; j < i; ++j) {
+            if (arc(S[j], S[i])) qp.bw[i] |= 1u << j;
+            if (arc(S[i], S[j])) qp.bwi[i] |= 1u << j;
+        }
+        bool starts = true;
+        for (uint32_t j = 0; j < i; ++j) starts = starts && comp[S[j]] != comp[S[i]];
+        const uint32_t nreq = __builtin_popcount(qp.bw[i]) + __builtin_popcount(qp.bwi[i]);
+        if (i > 0 && nreq == 0 && !starts)
+            return fail(ctx, CUTS_EINVAL, "order position %u (query vertex %u) has no backward neighbour", i, S[i]);
+        if (i > 0 && nreq > i)
+            return fail(ctx, CUTS_EUNSUPPORTED, "position %u needs %u lists (> %u): reciprocal query arcs at this position "
+                        "are not supported", i, nreq, i);
+    }
+    *out = qp;
+    return CUTS_OK;
+}
+
 // ---- kernel dispatch -------------------------------------------------------
 struct Window {
     uint64_t w0;
@@ -307,7 +386,7 @@ void launch_extend_nl(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t
 template <int J, int M>
 void launch_extend_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
-    const int nl = std::max(__builtin_popcount(ctx->q.bw[J]) - 1, 0);   // component root: 0
+    const int nl = std::max(__builtin_popcount(ctx->q.bw[J]) + __builtin_popcount(ctx->q.bwi[J]) - 1, 0);   // component root: 0
     switch (nl) {
         case 0: launch_extend_nl<J, 0, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
         case 1: if constexpr (J > 1) launch_extend_nl<J, (J > 1 ? 1 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
@@ -719,7 +798,7 @@ cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
     uint64_t off_canon, off_tmp;
     TRY(alloc_top(ctx, (uint64_t)ctx->n * 4 + 4, &off_canon));
     uint32_t* canon = (uint32_t*)(ctx->arena + off_canon);
-    DegAtLeast pred{ctx->deg, ctx->q.qdeg[0]};
+    DegAtLeast pred{ctx->deg, ctx->q.qdeg[0], ctx->directed ? ctx->n : 0u, ctx->q.qdin[0]};
     thrust::counting_iterator<uint32_t> it(0);
     size_t tmp_bytes = 0;
     unsigned long long* d_num = ctx->ctrl + kNumSel;
@@ -778,11 +857,11 @@ cuts_status build_free_lists(cuts_ctx* ctx, Run& r) {
     for (uint32_t J = 1; J < ctx->q.k; ++J) {
         ctx->q.foff[J] = 0;
         ctx->q.flen[J] = 0;
-        if (ctx->q.bw[J]) continue;
+        if (ctx->q.bw[J] | ctx->q.bwi[J]) continue;
         uint64_t off_list;
         TRY(alloc_bot(ctx, (uint64_t)ctx->n * 4 + 4, &off_list));
         const uint64_t top_save = ctx->top;
-        DegAtLeast pred{ctx->deg, ctx->q.qdeg[J]};
+        DegAtLeast pred{ctx->deg, ctx->q.qdeg[J], ctx->directed ? ctx->n : 0u, ctx->q.qdin[J]};
         thrust::counting_iterator<uint32_t> it(0);
         size_t tmp_bytes = 0;
         uint64_t off_tmp;
@@ -842,7 +921,11 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     r.enumerate = enumerate;
     r.rows = rows;
     r.cap_rows = cap_rows;
+    if (ctx->q_directed != ctx->directed)
+        return fail(ctx, CUTS_EINVAL, "%s query on a %s graph", ctx->q_directed ? "directed" : "undirected",
+                    ctx->directed ? "directed" : "undirected");
     r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words, ctx->colx};
+    r.g.dn = ctx->directed ? ctx->n : 0u;
     TRY(build_free_lists(ctx, r));
     uint64_t n1 = 0;
     const int k = (int)ctx->q.k;
@@ -912,6 +995,36 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
 
 }  // namespace
 
+namespace {
+cuts_status finish_query(cuts_ctx* ctx, const QPlan& qp, bool directed) {
+    ctx->q = qp;
+    ctx->q_directed = directed;
+    // ancestor-set reuse plan: deepest a in [2, J-1] with |bw[a]| >= 2 (an actual
+    // intersection), bw[a] a subset of bw[J] and deg_Q(S[a]) <= deg_Q(S[J])
+    // (undirected only)
+    ctx->need_ord = 0;
+    for (uint32_t J = 0; J <= kMaxK; ++J) ctx->anc[J] = 0;
+    for (uint32_t J = 3; J < qp.k && !directed; ++J)
+        for (uint32_t a = J - 1; a >= 2; --a)
+            if (__builtin_popcount(qp.bw[a]) >= 2 && (qp.bw[a] & ~qp.bw[J]) == 0 && qp.qdeg[a] <= qp.qdeg[J]) {
+                ctx->anc[J] = a;
+                ctx->need_ord |= 1u << a;
+                break;
+            }
+    ctx->root_begin = 0;
+    ctx->root_end = ~0ull;
+    ctx->slice_begin = 0;
+    ctx->slice_end = ~0ull;
+    ctx->part = 0;
+    ctx->nparts = 1;
+    ctx->pre_j = 0;
+    ctx->pre_count = 0;
+    ctx->pre_rows = nullptr;
+    ctx->has_query = true;
+    return CUTS_OK;
+}
+}  // namespace
+
 // ============================================================== C ABI
 extern "C" {
 
@@ -950,16 +1063,20 @@ void cuts_destroy(cuts_ctx* ctx) {
 
 const char* cuts_last_error(const cuts_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
 
-cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint64_t* d_row_ptr,
-                            const uint32_t* d_col, int validate) {
+namespace {
+cuts_status load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint64_t* d_row_ptr,
+                       const uint32_t* d_col, int validate, bool directed) {
     if (!ctx) return CUTS_EINVAL;
     ctx->err.clear();
     if (!d_row_ptr || (nnz && !d_col)) return fail(ctx, CUTS_EINVAL, "null graph pointer");
     if (n == 0xFFFFFFFFu) return fail(ctx, CUTS_EINVAL, "n must be < 2^32-1");
     CK(cudaSetDevice(ctx->device));
-    uint64_t deg_bytes = align_up((uint64_t)n * 4 + 4);
+    const uint64_t rows = directed ? 2ull * n : (uint64_t)n;   // directed: out-rows then in-rows
+    if (rows >= 0xFFFFFFFFull) return fail(ctx, CUTS_EINVAL, "2n must be < 2^32-1 for a directed graph");
+    uint64_t deg_bytes = align_up(rows * 4 + 4);
     if (kCtrlBytes + deg_bytes + (16u << 10) > ctx->arena_bytes) return fail(ctx, CUTS_ENOMEM, "arena too small for deg[%u]", n);
     ctx->has_graph = false;
+    ctx->directed = directed;
     ctx->n = n;
     ctx->nnz = nnz;
     ctx->row_ptr = d_row_ptr;
@@ -968,24 +1085,32 @@ cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint6
     ctx->base_off = kCtrlBytes + deg_bytes;
     if (n) {
         unsigned grid = (unsigned)std::min<uint64_t>(((uint64_t)n + 255) / 256, (uint64_t)ctx->num_sms * 8);
-        k_degree<<<grid, 256, 0, ctx->stream>>>(d_row_ptr, n, ctx->deg);
+        k_degree<<<grid, 256, 0, ctx->stream>>>(d_row_ptr, (uint32_t)rows, ctx->deg);
         CK(cudaGetLastError());
     }
     // row_ptr[0] == 0 and row_ptr[n] == nnz
     uint64_t ends[2] = {1, 0};
     CK(cudaMemcpyAsync(&ends[0], d_row_ptr, 8, cudaMemcpyDeviceToHost, ctx->stream));
-    CK(cudaMemcpyAsync(&ends[1], d_row_ptr + n, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(&ends[1], d_row_ptr + rows, 8, cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     if (ends[0] != 0 || ends[1] != nnz) return fail(ctx, CUTS_EINVAL, "row_ptr[0]=%llu row_ptr[n]=%llu nnz=%llu",
                                                     (unsigned long long)ends[0], (unsigned long long)ends[1], (unsigned long long)nnz);
     if (validate && n) {
         CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
         Graph g{d_row_ptr, d_col, ctx->deg, nullptr, nullptr, n, 0, nullptr};
-        unsigned grid = (unsigned)std::min<uint64_t>(((uint64_t)n * 32 + 255) / 256, (uint64_t)ctx->num_sms * 16);
+        g.dn = directed ? n : 0u;
+        unsigned grid = (unsigned)std::min<uint64_t>((rows * 32 + 255) / 256, (uint64_t)ctx->num_sms * 16);
         k_validate<<<grid, 256, 0, ctx->stream>>>(g, ctx->ctrl);
         CK(cudaGetLastError());
         TRY(read_ctrl(ctx));
-        if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_EINVAL, "graph is not canonical symmetric CSR (sorted, no loops/dups, ids < n)");
+        if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_EINVAL, directed ?
+            "digraph is not canonical (sorted, no loops/dups, ids < n, in-rows = transpose of out-rows)" :
+            "graph is not canonical symmetric CSR (sorted, no loops/dups, ids < n)");
+    }
+    if (directed) {   // hub bitmaps and the packed stream assume one symmetric row per vertex
+        ctx->nhubs = 0; ctx->hub_t_used = 0; ctx->hub = nullptr; ctx->bm = nullptr; ctx->colx = nullptr;
+        ctx->has_graph = true;
+        return CUTS_OK;
     }
     TRY(build_hubs(ctx));
     // packed candidate stream (degree filter without a gather) when ids fit 27 bits
@@ -1002,6 +1127,17 @@ cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint6
     ctx->has_graph = true;
     return CUTS_OK;
 }
+}  // namespace
+
+cuts_status cuts_load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint64_t* d_row_ptr,
+                            const uint32_t* d_col, int validate) {
+    return load_graph(ctx, n, nnz, d_row_ptr, d_col, validate, false);
+}
+
+cuts_status cuts_load_digraph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint64_t* d_row_ptr,
+                              const uint32_t* d_col, int validate) {
+    return load_graph(ctx, n, nnz, d_row_ptr, d_col, validate, true);
+}
 
 cuts_status cuts_set_hub_threshold(cuts_ctx* ctx, uint32_t t) {
     if (!ctx) return CUTS_EINVAL;
@@ -1017,30 +1153,20 @@ cuts_status cuts_set_query(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr, c
     QPlan qp{};
     ctx->has_query = false;
     TRY(plan_query(ctx, k, row_ptr, col, order, &qp));
-    ctx->q = qp;
-    // ancestor-set reuse plan: deepest a in [2, J-1] with |bw[a]| >= 2 (an actual
-    // intersection), bw[a] a subset of bw[J] and deg_Q(S[a]) <= deg_Q(S[J])
-    ctx->need_ord = 0;
-    for (uint32_t J = 0; J <= kMaxK; ++J) ctx->anc[J] = 0;
-    for (uint32_t J = 3; J < qp.k; ++J)
-        for (uint32_t a = J - 1; a >= 2; --a)
-            if (__builtin_popcount(qp.bw[a]) >= 2 && (qp.bw[a] & ~qp.bw[J]) == 0 && qp.qdeg[a] <= qp.qdeg[J]) {
-                ctx->anc[J] = a;
-                ctx->need_ord |= 1u << a;
-                break;
-            }
-    ctx->root_begin = 0;
-    ctx->root_end = ~0ull;
-    ctx->slice_begin = 0;
-    ctx->slice_end = ~0ull;
-    ctx->part = 0;
-    ctx->nparts = 1;
-    ctx->pre_j = 0;
-    ctx->pre_count = 0;
-    ctx->pre_rows = nullptr;
-    ctx->has_query = true;
-    return CUTS_OK;
+    return finish_query(ctx, qp, false);
 }
+
+cuts_status cuts_set_query_directed(cuts_ctx* ctx, uint32_t k, const uint32_t* row_ptr, const uint32_t* col,
+                                    const uint32_t* order) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (!ctx->has_graph) return fail(ctx, CUTS_ESTATE, "cuts_load_digraph must precede cuts_set_query_directed");
+    QPlan qp{};
+    ctx->has_query = false;
+    TRY(plan_query_directed(ctx, k, row_ptr, col, order, &qp));
+    return finish_query(ctx, qp, true);
+}
+
 
 cuts_status cuts_set_prefixes(cuts_ctx* ctx, uint32_t depth, uint64_t count, const uint32_t* d_prefixes) {
     if (!ctx) return CUTS_EINVAL;
@@ -1100,7 +1226,7 @@ cuts_status cuts_level1_size(cuts_ctx* ctx, uint64_t* canonical, uint64_t* in_ra
     ctx->top = ctx->arena_bytes & ~(kAlign - 1);
     uint64_t off_canon, off_tmp;
     TRY(alloc_top(ctx, (uint64_t)ctx->n * 4 + 4, &off_canon));
-    DegAtLeast pred{ctx->deg, ctx->q.qdeg[0]};
+    DegAtLeast pred{ctx->deg, ctx->q.qdeg[0], ctx->directed ? ctx->n : 0u, ctx->q.qdin[0]};
     thrust::counting_iterator<uint32_t> it(0);
     size_t tmp_bytes = 0;
     CK(cub::DeviceSelect::If(nullptr, tmp_bytes, it, (uint32_t*)(ctx->arena + off_canon), ctx->ctrl + kNumSel,

@@ -33,6 +33,12 @@ struct QPlan {                 // query in matching-order positions
     // sorted list at Graph::fre + foff[i] of flen[i] entries (built per run).
     uint64_t foff[kMaxK];
     uint32_t flen[kMaxK];
+    // directed Q (NEXT-1): bw[i] bit p <=> arc S[p] -> S[i] (candidate
+    // in children(f(S[p])), c-intersection); bwi[i] bit p <=> arc S[i] -> S[p]
+    // (candidate in parents(f(S[p])), p-intersection, Alg. 2 l.33-42).  qdeg is
+    // then the out-degree and qdin the in-degree (Def. 5 with P:262-264).
+    uint32_t bwi[kMaxK];
+    uint32_t qdin[kMaxK];
 };
 
 struct Trie {                  // lv[l] = level l (1-based): .x = data vertex, .y = parent index in level l-1
@@ -69,6 +75,7 @@ struct Graph {
     uint32_t words;
     const uint32_t* __restrict__ colx;  // col with min(deg, 31) packed in bits 27..31 (nullptr: n >= 2^27)
     const uint32_t* __restrict__ fre = nullptr;   // free lists of component roots (QPlan::foff/flen)
+    uint32_t dn = 0;   // directed: rows [0,n) are out-lists, rows [n,2n) in-lists, dn = n; undirected: 0
 };
 
 constexpr uint32_t kNoHub = 0xffffffffu;
@@ -164,20 +171,23 @@ __global__ void k_hub_fill(const uint64_t* __restrict__ row_ptr, const uint32_t*
     }
 }
 
-// graph validation: sorted strictly ascending rows, no loops, ids < n, symmetric.
-// one warp per vertex; sets ctrl[kErr] = 1 on any violation.
+// graph validation: sorted strictly ascending rows, no loops, ids < n, symmetric
+// (directed: the in-rows are the transpose of the out-rows).
+// one warp per row; sets ctrl[kErr] = 1 on any violation.
 __global__ void k_validate(Graph g, unsigned long long* ctrl) {
     const int lane = threadIdx.x & 31;
     const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t v = warp; v < g.n; v += nwarps) {
-        uint64_t b = g.row_ptr[v], e = g.row_ptr[v + 1];
+    for (uint64_t r = warp; r < (uint64_t)g.n + g.dn; r += nwarps) {
+        const uint64_t v = r < g.n ? r : r - g.n;
+        uint64_t b = g.row_ptr[r], e = g.row_ptr[r + 1];
         bool bad = e < b;
         for (uint64_t p = b + lane; !bad && p < e; p += 32) {
             uint32_t u = g.col[p];
             if (u >= g.n || u == v) { bad = true; break; }
             if (p > b && g.col[p - 1] >= u) { bad = true; break; }
-            if (!list_contains(g.col, g.row_ptr[u], g.row_ptr[u + 1], (uint32_t)v)) { bad = true; break; }
+            const uint64_t o = r < g.n ? (uint64_t)u + g.dn : (uint64_t)u;   // the opposite row of u
+            if (!list_contains(g.col, g.row_ptr[o], g.row_ptr[o + 1], (uint32_t)v)) { bad = true; break; }
         }
         if (__any_sync(0xffffffffu, bad) && lane == 0) atomicExch(ctrl + kErr, 1ull);
     }
@@ -185,9 +195,9 @@ __global__ void k_validate(Graph g, unsigned long long* ctrl) {
 
 // ---------------------------------------------------------------- level 1
 // canonical level-1 flags: deg(v) >= deg_Q(S[0])  (Alg. 1 l.8-11)
-struct DegAtLeast {
-    const uint32_t* deg; uint32_t t;
-    __host__ __device__ bool operator()(uint32_t v) const { return deg[v] >= t; }
+struct DegAtLeast {   // directed: deg[v] = out-degree, deg[dn + v] = in-degree
+    const uint32_t* deg; uint32_t t; uint32_t dn = 0; uint32_t ti = 0;
+    __host__ __device__ bool operator()(uint32_t v) const { return deg[v] >= t && (ti == 0 || deg[dn + v] >= ti); }
 };
 
 // seeded bijection on [0, R) (4-round Feistel + cycle walking): the randomised
@@ -251,6 +261,8 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                                               uint32_t* __restrict__ lst_len,
                                               unsigned long long* __restrict__ ctrl, int count_bytes, Reuse ru) {
     const uint32_t bw = q.bw[J];
+    const uint32_t bwi = q.bwi[J];
+    constexpr int J2 = 2 * J;   // list slots: [0, J) children of path[p], [J, 2J) parents (directed)
     unsigned long long bytes_plan = 0, bytes_ext = 0;
     for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e <= W; e += gridDim.x * blockDim.x) {
         if (e == W) { ub[W] = 0; continue; }
@@ -266,27 +278,29 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
             path[p] = cur.x;
             idx = cur.y;
         }
-        uint64_t lb_[J];
-        uint32_t ln_[J];
+        uint64_t lb_[J2];
+        uint32_t ln_[J2];
         uint64_t lists = 0, best_b = 0;
         uint32_t best_d = 0xffffffffu;
         int best = -1;
+        const uint32_t need = bw | (bwi << J);
 #pragma unroll
-        for (int p = 0; p < J; ++p) {
-            ln_[p] = 0xffffffffu;
-            lb_[p] = 0;
-            if ((bw >> p) & 1u) {
-                const uint64_t b = g.row_ptr[path[p]];
-                const uint32_t d = (uint32_t)(g.row_ptr[path[p] + 1] - b);
+        for (int s = 0; s < J2; ++s) {
+            ln_[s] = 0xffffffffu;
+            lb_[s] = 0;
+            if ((need >> s) & 1u) {
+                const uint64_t row = s < J ? (uint64_t)path[s] : (uint64_t)path[s - J] + g.dn;
+                const uint64_t b = g.row_ptr[row];
+                const uint32_t d = (uint32_t)(g.row_ptr[row + 1] - b);
                 lists += d;
-                lb_[p] = b;
-                ln_[p] = d;
-                if (best < 0 || d < best_d) { best = p; best_d = d; best_b = b; }
+                lb_[s] = b;
+                ln_[s] = d;
+                if (best < 0 || d < best_d) { best = s; best_d = d; best_b = b; }
             }
         }
         // ancestor-set source: the children range of the level-a ancestor replaces
         // the lists of bw[a] when it is no longer than every remaining list
-        uint32_t keep = bw;                          // lists still to be tested
+        uint32_t keep = need;                        // lists still to be tested
         bool trie = false;
         uint64_t trie_off = 0, rest_sum = 0;
         uint32_t trie_len = 0;
@@ -301,7 +315,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                 if (((bw & ~ru.bwa) >> p) & 1u) { rest_min = min(rest_min, ln_[p]); rest_sum += ln_[p]; }
             if (trie_len <= rest_min) { trie = true; keep = bw & ~ru.bwa; }
         }
-        if (bw == 0) {           // component root: cross-product factor
+        if (need == 0) {         // component root: cross-product factor
             src_off[e] = q.foff[J] | kFreeSrc;
             ub[e] = q.flen[J];
             lists = q.flen[J];
@@ -316,23 +330,24 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         // other lists: hub rows become bitmap probes; then sort by length
         int x = 0;
 #pragma unroll
-        for (int p = 0; p < J; ++p) {
+        for (int p = 0; p < J2; ++p) {
             if (p != best && ((keep >> p) & 1u)) {
-                const uint32_t h = g.hub ? __ldg(g.hub + path[p]) : kNoHub;
+                // hub bitmaps cover out-rows of an undirected graph only (g.hub is null when directed)
+                const uint32_t h = (g.hub && p < J) ? __ldg(g.hub + path[p]) : kNoHub;
                 if (h != kNoHub) { lb_[p] = (uint64_t)h * g.words; ln_[p] |= kBmFlag; }
             } else {
                 ln_[p] = 0xffffffffu;     // not a list to test (the source, or not backward)
             }
         }
 #pragma unroll
-        for (int i = 0; i < J; ++i)
+        for (int i = 0; i < J2; ++i)
 #pragma unroll
-            for (int y = 0; y + 1 < J - i; ++y)
+            for (int y = 0; y + 1 < J2 - i; ++y)
                 if (ln_[y + 1] < ln_[y]) {
                     const uint32_t tl = ln_[y]; ln_[y] = ln_[y + 1]; ln_[y + 1] = tl;
                     const uint64_t tb = lb_[y]; lb_[y] = lb_[y + 1]; lb_[y + 1] = tb;
                 }
-        const int nl = __popc(bw) - 1;   // -1 for a component root: no lists
+        const int nl = __popc(need) - 1;   // -1 for a component root: no lists (host: nl <= J-1)
 #pragma unroll
         for (int y = 0; y < J - 1; ++y)
             if (y < nl) {
@@ -343,7 +358,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
 #pragma unroll
         for (int p = 0; p < J; ++p) path_s[(size_t)p * W + e] = path[p];
         if (count_bytes) {   // 8 (entry) + 8(J-1) (hops) + 16 per list bound
-            bytes_plan += 8ull + 8ull * (J - 1) + 16ull * __popc(bw);
+            bytes_plan += 8ull + 8ull * (J - 1) + 16ull * __popc(need);
             if (trie) {          // the ancestor range (8 B entries) + the lists not covered by it
                 bytes_ext += 8ull * trie_len + 4ull * rest_sum;
             } else {
@@ -416,6 +431,10 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
     const int vl = lane & (G - 1);
     const int vb = lane & ~(G - 1);
     const uint32_t qd = q.qdeg[J];
+    const uint32_t qdi = q.qdin[J];              // directed: in-degree bound (0: none)
+    // undirected: a candidate from a list has deg >= 1, so qdeg <= 1 needs no check;
+    // directed: a child may have out-degree 0
+    const uint32_t qmin = g.dn ? 0u : 1u;
     unsigned long long my_count = 0, bytes = 0;
     unsigned int* work = (unsigned int*)(ctrl + kWork);
     const unsigned long long wbytes = M == kCount ? 0ull : (M == kEnum ? 4ull * q.k : 8ull);
@@ -463,13 +482,13 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
             // a component root's free list is already degree-filtered
             const bool fsrc = (so & kFreeSrc) != 0;
             // packed CSR source (degree in the id word) only where a degree filter applies
-            const bool pk = !tsrc && !fsrc && g.colx != nullptr && qd > 1;
+            const bool pk = !tsrc && !fsrc && g.colx != nullptr && qd > qmin;
             const uint32_t* __restrict__ src = tsrc ? (const uint32_t*)(rsrc + (so & ~kTrieSrc))
                                              : fsrc ? g.fre + (so & ~kFreeSrc) : (pk ? g.colx : g.col) + so;
             const uint32_t ssh = tsrc ? 1u : 0u;
             const uint32_t umask = pk ? kPackMask : 0xffffffffu;
             // an ancestor range already passed deg >= qdeg[a]: no check needed when qdeg[J] <= qdeg[a]
-            const bool dload = qd > 1 && !pk && !fsrc && !(tsrc && qd <= qda);
+            const bool dload = qd > qmin && !pk && !fsrc && !(tsrc && qd <= qda);
             const uint32_t nit = (ihi - ilo + G - 1) / G;
             unsigned long long ecnt = 0, run = 0;   // per-entry count (pass A) / ordered-write cursor
             uint32_t nit_max = nit;
@@ -521,7 +540,11 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                     bool k0 = a0, k1 = a1;
 #pragma unroll
                     for (int p = 0; p < J; ++p) { k0 = k0 && (path[p] != c0); k1 = k1 && (path[p] != c1); }
-                    if (qd > 1) {
+                    if (qdi) {
+                        k0 = k0 && __ldg(g.deg + g.dn + c0) >= qdi;
+                        k1 = k1 && __ldg(g.deg + g.dn + c1) >= qdi;
+                    }
+                    if (qd > qmin) {
                         const uint32_t d0 = pk ? (r0 >> kPackShift) : ((k0 && dload) ? __ldg(g.deg + c0) : 0xffffffffu);
                         const uint32_t d1 = pk ? (r1 >> kPackShift) : ((k1 && dload) ? __ldg(g.deg + c1) : 0xffffffffu);
                         k0 = k0 && d0 >= qd;
@@ -549,6 +572,7 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                 for (int x = 0; x < NL; ++x)
                     bmw[x] = (pre && (ln[x] & kBmFlag) && ln[x] != kSkip) ? __ldg(lb[x] + (c >> 5)) : 0xffffffffu;
                 bool ok = inj && dg >= qd;                                    // every neighbour has deg >= 1
+                if (qdi) ok = ok && __ldg(g.deg + g.dn + c) >= qdi;          // directed: in-degree
                 bool inter = count_bytes ? act : ok;
 #pragma unroll
                 for (int x = 0; x < NL; ++x)                                  // c-intersection (Alg. 2): hubs
