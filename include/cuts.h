@@ -99,6 +99,8 @@ typedef struct {
                                   mode never uses it                                        */
 #define CUTS_DEBUG_NO_PACK  8u /* at the next cuts_load_graph: no packed (id | degree) copy
                                   of col in the arena (ablation)                            */
+#define CUTS_DEBUG_FIRST_SOURCE 16u /* ablation (NEXT-2): stream the FIRST backward list as
+                                  Alg. 2 l.22-23 does (a1) instead of the shortest one      */
 
 /* Create a context bound to opts->device / opts->stream / opts->arena.
  * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */

@@ -39,6 +39,7 @@ struct QPlan {                 // query in matching-order positions
     // then the out-degree and qdin the in-degree (Def. 5 with P:262-264).
     uint32_t bwi[kMaxK];
     uint32_t qdin[kMaxK];
+    uint32_t src_first;        // ablation: source = first backward list (Alg. 2 a1), not the shortest
 };
 
 struct Trie {                  // lv[l] = level l (1-based): .x = data vertex, .y = parent index in level l-1
@@ -295,7 +296,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                 lists += d;
                 lb_[s] = b;
                 ln_[s] = d;
-                if (best < 0 || d < best_d) { best = s; best_d = d; best_b = b; }
+                if (best < 0 || (!q.src_first && d < best_d)) { best = s; best_d = d; best_b = b; }
             }
         }
         // ancestor-set source: the children range of the level-a ancestor replaces

@@ -136,6 +136,31 @@ def test_packed_degree_stream_ablation(cuts):
     c.set_debug()
 
 
+def test_first_source_ablation(cuts):
+    """NEXT-2 ablation: streaming the FIRST backward list (Alg. 2's a1,
+    CUTS_DEBUG_FIRST_SOURCE) instead of the shortest gives the same counts,
+    level sizes and rows, with and without hubs and reuse."""
+    g = rmat_graph(9, 8, a=0.55, b=0.2, c=0.2, seed=6)
+    c = cuts(device=0, arena_bytes=1 << 20)
+    for hub in (None, 0):
+        c.set_hub_threshold(hub)
+        c.load_csr(g)
+        for q in DENSE5[::2] + SPARSE5[::3] + dense_family(6)[::4]:
+            want, lv = oracle.count(g, q, levels=True)
+            _set(c, q)
+            for kw in ({"first_source": True}, {"first_source": True, "no_reuse": True}):
+                c.set_debug(**kw)
+                assert c.count("hybrid") == want, (hub, q.name, kw)
+                assert c.stats()["level_size"] == lv, (hub, q.name, kw)
+        c.set_debug(first_source=True)
+        q = DENSE5[5]
+        want = oracle.count(g, q)
+        _set(c, q)
+        if want <= 2_000_000:
+            assert np.array_equal(_sorted_rows(c.enumerate("hybrid", cap_rows=want)), oracle.enumerate_rows(g, q))
+        c.set_debug()
+
+
 def test_ancestor_reuse_enumerate(ctx):
     g = er_graph(40, 420, 7)
     ctx.load_csr(g)

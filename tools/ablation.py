@@ -1,0 +1,89 @@
+"""NEXT-2 intersection-method ablation on one GPU.
+
+    python tools/ablation.py --workload C2 [--reps 2] [--out f.jsonl]
+
+Per (graph, query) and variant, best-of-reps seconds of cuts_count plus the
+k_extend milliseconds.  Variants (all give the same counts; checked here):
+  paper_c   : the paper's c-intersection (Alg. 2 l.19-31): the FIRST backward
+              list a1 is the candidate stream, membership by binary search;
+              no hub bitmaps, no packed degree stream, no ancestor source
+  short_c   : as paper_c, but the SHORTEST list is the stream (B200 choice)
+  sv_hubs   : + SV-style bitmaps for hub lists (Alg. 2 l.7-17)
+  packed    : + packed (id | degree) stream (degree filter without a gather)
+  full      : + ancestor-set source (the product default)
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from workloads import WORKLOADS  # noqa: E402
+from paper_conf_sc_xiangkshs21_b200 import Cuts  # noqa: E402
+
+VARIANTS = [  # (name, hub threshold, debug kwargs)
+    ("paper_c", None, dict(first_source=True, no_pack=True, no_reuse=True)),
+    ("short_c", None, dict(no_pack=True, no_reuse=True)),
+    ("sv_hubs", 0, dict(no_pack=True, no_reuse=True)),
+    ("packed", 0, dict(no_reuse=True)),
+    ("full", 0, dict()),
+]
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="C2")
+    ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--variants", default=",".join(v[0] for v in VARIANTS))
+    ap.add_argument("--query", default="")
+    ap.add_argument("--out", default="")
+    args = ap.parse_args()
+    wl = WORKLOADS[args.workload]
+    ctx = Cuts(device=0)
+    want = {}
+    totals = {}
+    for name, hub, dbg in VARIANTS:
+        if name not in args.variants.split(","):
+            continue
+        totals[name] = 0.0
+        for spec, qs in wl.parts:
+            g = spec.build()
+            ctx.set_hub_threshold(hub)
+            ctx.set_debug(**dbg)          # NO_PACK acts at load
+            ctx.load_csr(g)
+            for q in qs:
+                if args.query and q.name != args.query:
+                    continue
+                qr, qc = q.csr()
+                ctx.set_query(qr, qc)
+                ctx.set_debug(timing=True, **dbg)
+                best, st, c = None, None, None
+                for _ in range(args.reps):
+                    torch.cuda.synchronize()
+                    t = time.time()
+                    c = ctx.count(wl.mode)
+                    dt = time.time() - t
+                    if best is None or dt < best:
+                        best, st = dt, ctx.stats()
+                key = (spec.name, q.name)
+                assert want.setdefault(key, c) == c, (name, key, c, want[key])
+                totals[name] += best
+                rec = {"variant": name, "graph": spec.name, "query": q.name, "count": c, "s": round(best, 4),
+                       "ms_extend": round(st["ms_extend"], 2), "ms_plan": round(st["ms_plan"], 2),
+                       "hubs": st["hubs"], "items": st["items"]}
+                line = json.dumps(rec)
+                print(line, flush=True)
+                if args.out:
+                    with open(args.out, "a") as f:
+                        f.write(line + "\n")
+        print(json.dumps({"variant": name, "total_s": round(totals[name], 3)}), flush=True)
+    ctx.set_debug()
+
+
+if __name__ == "__main__":
+    main()
