@@ -101,6 +101,9 @@ typedef struct {
                                   of col in the arena (ablation)                            */
 #define CUTS_DEBUG_FIRST_SOURCE 16u /* ablation (NEXT-2): stream the FIRST backward list as
                                   Alg. 2 l.22-23 does (a1) instead of the shortest one      */
+#define CUTS_DEBUG_NO_FAST_COUNT 32u /* ablation: stream the list at a single-list,
+                                  degree-free last level of cuts_count instead of counting
+                                  |list| - |path found in list| by binary search            */
 
 /* Create a context bound to opts->device / opts->stream / opts->arena.
  * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */

@@ -229,10 +229,10 @@ class Cuts:
         return int(a.value), int(b.value)
 
     def set_debug(self, timing: bool = False, bytes_: bool = False, no_reuse: bool = False,
-                  no_pack: bool = False, first_source: bool = False):
+                  no_pack: bool = False, first_source: bool = False, no_fast_count: bool = False):
         """CUTS_DEBUG_* flags: instrumentation and the NEXT-2 ablations (include/cuts.h)."""
         flags = ((1 if timing else 0) | (2 if bytes_ else 0) | (4 if no_reuse else 0) |
-                 (8 if no_pack else 0) | (16 if first_source else 0))
+                 (8 if no_pack else 0) | (16 if first_source else 0) | (32 if no_fast_count else 0))
         self._check(self.lib.cuts_set_debug(self.h, flags))
         return self
 

@@ -927,6 +927,7 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words, ctx->colx};
     r.g.dn = ctx->directed ? ctx->n : 0u;
     ctx->q.src_first = (ctx->debug & CUTS_DEBUG_FIRST_SOURCE) ? 1u : 0u;
+    ctx->q.count_fast = (!enumerate && !(ctx->debug & CUTS_DEBUG_NO_FAST_COUNT)) ? 1u : 0u;
     TRY(build_free_lists(ctx, r));
     uint64_t n1 = 0;
     const int k = (int)ctx->q.k;

@@ -40,7 +40,17 @@ struct QPlan {                 // query in matching-order positions
     uint32_t bwi[kMaxK];
     uint32_t qdin[kMaxK];
     uint32_t src_first;        // ablation: source = first backward list (Alg. 2 a1), not the shortest
+    uint32_t count_fast;       // cuts_count: set-difference count at a single-list last level
 };
+
+// Count-only last level with ONE backward list and no degree bound:
+// the children of an entry are list \ path, so their number is |list| minus the
+// path vertices found in the list (<= J binary searches) — the exact size of the
+// intersection result without streaming the list.
+template <int J>
+__device__ __forceinline__ bool fast_last(const QPlan& q, uint32_t need, uint32_t qmin) {
+    return q.count_fast && J + 1 == (int)q.k && __popc(need) == 1 && q.qdeg[J] <= qmin && q.qdin[J] == 0;
+}
 
 struct Trie {                  // lv[l] = level l (1-based): .x = data vertex, .y = parent index in level l-1
     const uint2* lv[kMaxK];
@@ -362,6 +372,8 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
             bytes_plan += 8ull + 8ull * (J - 1) + 16ull * __popc(need);
             if (trie) {          // the ancestor range (8 B entries) + the lists not covered by it
                 bytes_ext += 8ull * trie_len + 4ull * rest_sum;
+            } else if (fast_last<J>(q, need, g.dn ? 0u : 1u)) {   // J binary searches in the list
+                bytes_ext += 4ull * J * (32 - __clz(best_d));
             } else {
                 bytes_ext += 4ull * lists;               // every backward list read once
             }
@@ -527,7 +539,30 @@ __global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend
                     }
                 }
             };
-            if constexpr (NL == 0) {
+            bool fast = false;
+            if constexpr (NL == 0 && M == kCount) fast = !tsrc && !fsrc && fast_last<J>(q, q.bw[J] | (q.bwi[J] << J), qmin);
+            if (fast) {
+                // |list[ilo, ihi) \ path|: lane vl < J looks for path[vl] (a distinct vertex)
+                if (has) {
+                    unsigned long long c = vl == 0 ? (unsigned long long)(ihi - ilo) : 0ull;
+                    if (vl < J && ihi > ilo) {
+                        uint32_t x = path[0];
+#pragma unroll
+                        for (int p = 1; p < J; ++p) x = (p == vl) ? path[p] : x;
+                        const uint32_t* b0 = src + ilo;
+                        uint32_t len = ihi - ilo;
+                        while (len > 1) {
+                            const uint32_t half = len >> 1;
+                            b0 = (__ldg(b0 + half - 1) < x) ? b0 + half : b0;
+                            len -= half;
+                        }
+                        if (__ldg(b0) == x) c -= 1ull;    // u64 wrap: the warp sum is exact
+                        if (count_bytes) bytes += 4ull * (32 - __clz(ihi - ilo));
+                    }
+                    my_count += c;
+                    ecnt += c;
+                }
+            } else if constexpr (NL == 0) {
                 // one backward list: it is the source, so the intersection is the list
                 // itself and only injectivity + degree remain; two candidates per lane per
                 // iteration, loads issued together

@@ -161,6 +161,27 @@ def test_first_source_ablation(cuts):
         c.set_debug()
 
 
+@pytest.mark.parametrize("arena_kib", [64, 1024])
+def test_fast_last_level_count(cuts, arena_kib):
+    """Single-list degree-free last level of cuts_count (|list| - path vertices
+    found by binary search) against the oracle and against the streamed list
+    (CUTS_DEBUG_NO_FAST_COUNT), incl. hybrid chunks that split an entry's list."""
+    g = rmat_graph(9, 8, a=0.55, b=0.2, c=0.2, seed=8)
+    c = cuts(device=0, arena_bytes=arena_kib << 10)
+    c.load_csr(g)
+    qs = [q for q in SPARSE5 if q.name in ("P5", "K1_4", "chair", "bull", "cricket")]
+    qs += [named_query(x) for x in ("P3", "P4", "S3", "K2")] + [query_from_edges(4, [(0, 1), (1, 2), (0, 2), (2, 3)])]
+    for q in qs:
+        want, lv = oracle.count(g, q, levels=True)
+        _set(c, q)
+        for kw in ({}, {"no_fast_count": True}):
+            c.set_debug(**kw)
+            for mode in ("hybrid", "bfs") if arena_kib > 64 else ("hybrid",):
+                assert c.count(mode) == want, (q.name, kw, mode)
+                assert c.stats()["level_size"] == lv, (q.name, kw, mode)
+    c.set_debug()
+
+
 def test_ancestor_reuse_enumerate(ctx):
     g = er_graph(40, 420, 7)
     ctx.load_csr(g)
