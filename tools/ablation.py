@@ -10,7 +10,9 @@ k_extend milliseconds.  Variants (all give the same counts; checked here):
   short_c   : as paper_c, but the SHORTEST list is the stream (B200 choice)
   sv_hubs   : + SV-style bitmaps for hub lists (Alg. 2 l.7-17)
   packed    : + packed (id | degree) stream (degree filter without a gather)
-  full      : + ancestor-set source (the product default)
+  reuse     : + ancestor-set source
+  full      : + set-difference count at a single-list degree-free last level
+              (the product default)
 """
 import argparse
 import json
@@ -27,10 +29,11 @@ from workloads import WORKLOADS  # noqa: E402
 from paper_conf_sc_xiangkshs21_b200 import Cuts  # noqa: E402
 
 VARIANTS = [  # (name, hub threshold, debug kwargs)
-    ("paper_c", None, dict(first_source=True, no_pack=True, no_reuse=True)),
-    ("short_c", None, dict(no_pack=True, no_reuse=True)),
-    ("sv_hubs", 0, dict(no_pack=True, no_reuse=True)),
-    ("packed", 0, dict(no_reuse=True)),
+    ("paper_c", None, dict(first_source=True, no_pack=True, no_reuse=True, no_fast_count=True)),
+    ("short_c", None, dict(no_pack=True, no_reuse=True, no_fast_count=True)),
+    ("sv_hubs", 0, dict(no_pack=True, no_reuse=True, no_fast_count=True)),
+    ("packed", 0, dict(no_reuse=True, no_fast_count=True)),
+    ("reuse", 0, dict(no_fast_count=True)),
     ("full", 0, dict()),
 ]
 
