@@ -409,7 +409,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
 // (dropped past cap; HYBRID sizes cap so that never happens); kCount -> 128-bit
 // count; kEnum -> rows of k u32 in query-id order at ctrl[kEnumCursor].
 template <int J, int NL, int M, int G>
-__global__ void __launch_bounds__(256, (J <= 3) ? 6 : (J <= 5 ? 5 : 4)) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
+__global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J <= 5 ? 5 : 4)) k_extend(Graph g, QPlan q, uint64_t w0, uint32_t W,
                                                const uint32_t* __restrict__ path_s,
                                                const uint64_t* __restrict__ src_off,
                                                const uint64_t* __restrict__ offs,

