@@ -161,7 +161,7 @@ def test_first_source_ablation(cuts):
         c.set_debug()
 
 
-@pytest.mark.parametrize("arena_kib", [64, 1024])
+@pytest.mark.parametrize("arena_kib", [64, 256 << 10])
 def test_fast_last_level_count(cuts, arena_kib):
     """Single-list degree-free last level of cuts_count (|list| - path vertices
     found by binary search) against the oracle and against the streamed list
