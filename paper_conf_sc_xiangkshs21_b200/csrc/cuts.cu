@@ -333,7 +333,11 @@ struct Window {
 
 template <int J>
 void launch_plan_t(cuts_ctx* ctx, const Graph& g, const Trie& t, const Window& w, int grid) {
-    k_plan<J><<<grid, 256, 0, ctx->stream>>>(g, t, ctx->q, w.w0, w.W, w.path, w.src, w.ub, w.lst_off, w.lst_len, ctx->ctrl,
+    if (ctx->directed)
+        k_plan<J, true><<<grid, 256, 0, ctx->stream>>>(g, t, ctx->q, w.w0, w.W, w.path, w.src, w.ub, w.lst_off, w.lst_len, ctx->ctrl,
+                                             (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0, w.ru);
+    else
+        k_plan<J, false><<<grid, 256, 0, ctx->stream>>>(g, t, ctx->q, w.w0, w.W, w.path, w.src, w.ub, w.lst_off, w.lst_len, ctx->ctrl,
                                              (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0, w.ru);
 }
 

@@ -263,7 +263,7 @@ __global__ void k_rows_k1(const uint2* __restrict__ L1, uint64_t cnt, uint32_t* 
 // recomputing them lane-redundantly.
 //   lst_off[x*W + e]: element offset into col (or into bm for a bitmap row)
 //   lst_len[x*W + e]: list length, | kBmFlag for a bitmap row
-template <int J>
+template <int J, bool D>
 __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t w0, uint32_t W,
                                               uint32_t* __restrict__ path_s,
                                               uint64_t* __restrict__ src_off,
@@ -273,7 +273,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
                                               unsigned long long* __restrict__ ctrl, int count_bytes, Reuse ru) {
     const uint32_t bw = q.bw[J];
     const uint32_t bwi = q.bwi[J];
-    constexpr int J2 = 2 * J;   // list slots: [0, J) children of path[p], [J, 2J) parents (directed)
+    constexpr int J2 = D ? 2 * J : J;   // list slots: [0, J) children of path[p], [J, 2J) parents (directed)
     unsigned long long bytes_plan = 0, bytes_ext = 0;
     for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e <= W; e += gridDim.x * blockDim.x) {
         if (e == W) { ub[W] = 0; continue; }
@@ -294,7 +294,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         uint64_t lists = 0, best_b = 0;
         uint32_t best_d = 0xffffffffu;
         int best = -1;
-        const uint32_t need = bw | (bwi << J);
+        const uint32_t need = D ? (bw | (bwi << J)) : bw;
 #pragma unroll
         for (int s = 0; s < J2; ++s) {
             ln_[s] = 0xffffffffu;
