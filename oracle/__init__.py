@@ -31,7 +31,7 @@ class OracleError(RuntimeError):
 def build(force: bool = False) -> str:
     """Compile the oracle with gcc (plain -O2; no tuning)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-o", _LIB, _SRC])
+        subprocess.check_call(["gcc", "-O2", "-std=gnu11", "-shared", "-fPIC", "-pthread", "-o", _LIB, _SRC])
     return _LIB
 
 
@@ -53,6 +53,12 @@ def _load():
         lib.oracle_di_count.argtypes = [ctypes.c_uint32, u64p, u32p, u64p, u32p, ctypes.c_uint32, u32p, u32p,
                                         u32p, u64p, u64p, u64p, u64p, u32p, ctypes.c_uint64]
         lib.oracle_di_order.argtypes = [ctypes.c_uint32, u32p, u32p, u32p]
+        lib.oracle_cross_product.argtypes = [ctypes.c_uint32, ctypes.c_uint32, u32p, ctypes.POINTER(u32p),
+                                             ctypes.POINTER(u32p), u64p, u32p, ctypes.c_uint64, u64p, u64p]
+        lib.oracle_count_mt.argtypes = [ctypes.c_uint32, ctypes.c_uint32, u64p, u32p, ctypes.c_uint32, u32p, u32p,
+                                        u32p, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, u64p, u64p]
+        lib.oracle_cross_product.restype = ctypes.c_int
+        lib.oracle_count_mt.restype = ctypes.c_int
         lib.oracle_di_count.restype = ctypes.c_int
         lib.oracle_di_order.restype = ctypes.c_int
         for f in (lib.oracle_count, lib.oracle_enumerate, lib.oracle_order,
@@ -148,35 +154,44 @@ class _SubQuery:
         return row, np.asarray([v for a in adj for v in a], dtype=np.uint32)
 
 
-def _cross_product_rows(g, q) -> np.ndarray:
+def _cross_product(g, q, want_rows: bool):
     """P:546-551 step by step: per-component embeddings (the connected oracle
-    below), then their cross product, keeping injective combinations only."""
+    below, each component as its own query), then their cross product keeping
+    injective combinations only — nested loops in C (``oracle_cross_product``),
+    nothing materialised but the component rows.  Returns (count, rows|None)."""
     comps = components(q)
-    rows = np.zeros((1, q.k), dtype=np.uint32)      # the empty partial map
-    placed = []
-    for comp in comps:
-        sub = enumerate_rows(g, _sub_query(q, comp))
-        if rows.shape[0] == 0 or sub.shape[0] == 0:
-            return np.zeros((0, q.k), dtype=np.uint32)
-        a = np.repeat(rows, sub.shape[0], axis=0)
-        b = np.tile(sub, (rows.shape[0], 1))
-        ok = np.ones(a.shape[0], dtype=bool)
-        for x in placed:                              # injectivity across components
-            for y in range(len(comp)):
-                ok &= a[:, x] != b[:, y]
-        a = a[ok]
-        a[:, comp] = b[ok]
-        rows = a
-        placed.extend(comp)
-    order_ = np.lexsort(rows.T[::-1])
-    return rows[order_]
+    subs = [enumerate_rows(g, _sub_query(q, comp)) for comp in comps]
+    nc = len(comps)
+    sizes = np.array([len(c) for c in comps], dtype=np.uint32)
+    verts = [np.ascontiguousarray(c, dtype=np.uint32) for c in comps]
+    crow = [np.ascontiguousarray(s if s.size else np.zeros((1, len(c)), np.uint32), dtype=np.uint32)
+            for s, c in zip(subs, comps)]
+    ccount = np.array([s.shape[0] for s in subs], dtype=np.uint64)
+    u32p = ctypes.POINTER(ctypes.c_uint32)
+    va = (u32p * nc)(*[_p(v, ctypes.c_uint32) for v in verts])
+    ra = (u32p * nc)(*[_p(r, ctypes.c_uint32) for r in crow])
+    lo, hi = np.zeros(1, np.uint64), np.zeros(1, np.uint64)
+    lib = _load()
+
+    def call(rows, cap):
+        _check(lib.oracle_cross_product(q.k, nc, _p(sizes, ctypes.c_uint32), va, ra, _p(ccount, ctypes.c_uint64),
+                                        None if rows is None else _p(rows, ctypes.c_uint32), cap,
+                                        _p(lo, ctypes.c_uint64), _p(hi, ctypes.c_uint64)))
+        return int(lo[0]) | (int(hi[0]) << 64)
+
+    n = call(None, 0)
+    if not want_rows:
+        return n, None
+    rows = np.zeros((max(n, 1), q.k), dtype=np.uint32)
+    call(rows, n)
+    return n, rows[:n]
 
 
 def count(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 - 1, levels: bool = False):
     """Exact number of ordered non-induced embeddings (Python int, 128-bit).
 
     A disconnected Q goes through the per-component cross product of P:546-551
-    (``_cross_product_rows``; no order, root range or level sizes there).
+    (``_cross_product``; no order, root range or level sizes there).
 
     With ``levels=True`` returns ``(count, [|L_0|, |L_1|, ..., |L_k|])`` where
     |L_j| counts partial paths of j matched vertices (|L_0| is 0).
@@ -184,7 +199,7 @@ def count(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 - 1, leve
     if len(components(q)) > 1:
         if order is not None or root_begin != 0 or root_end != 2**64 - 1 or levels:
             raise OracleError(ORC_EUNSUPPORTED)
-        return int(_cross_product_rows(g, q).shape[0])
+        return _cross_product(g, q, False)[0]
     rp, col = _graph_arrays(g)
     qr, qc, o = _query_arrays(q, order)
     lo = np.zeros(1, np.uint64)
@@ -209,7 +224,7 @@ def enumerate_rows(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 
     if len(components(q)) > 1:
         if order is not None or root_begin != 0 or root_end != 2**64 - 1:
             raise OracleError(ORC_EUNSUPPORTED)
-        rows = _cross_product_rows(g, q)
+        rows = _cross_product(g, q, True)[1]
         return rows if cap_rows is None else rows[:cap_rows]
     if cap_rows is None:
         cap_rows = count(g, q, order, root_begin, root_end)
@@ -224,6 +239,21 @@ def enumerate_rows(g, q, order=None, root_begin: int = 0, root_end: int = 2**64 
                                   _p(nf, ctypes.c_uint64))
     _check(rc)
     return rows[:min(int(nf[0]), cap_rows)]
+
+
+def count_mt(g, q, threads: int, root_begin: int = 0, root_end: int = 2**64 - 1, grain: int = 1,
+             order=None) -> int:
+    """Root-parallel driver (``oracle_count_mt``): the same ``rec`` on disjoint
+    canonical root ranges pulled by `threads` pthreads, summed.  Used for the
+    N-core CPU baseline only; parity pins use ``count``."""
+    rp, col = _graph_arrays(g)
+    qr, qc, o = _query_arrays(q, order)
+    lo, hi = np.zeros(1, np.uint64), np.zeros(1, np.uint64)
+    _check(_load().oracle_count_mt(threads, g.n, _p(rp, ctypes.c_uint64), _p(col, ctypes.c_uint32), q.k,
+                                   _p(qr, ctypes.c_uint32), _p(qc, ctypes.c_uint32),
+                                   None if o is None else _p(o, ctypes.c_uint32), root_begin, root_end, grain,
+                                   _p(lo, ctypes.c_uint64), _p(hi, ctypes.c_uint64)))
+    return int(lo[0]) | (int(hi[0]) << 64)
 
 
 def level1_size(g, min_deg: int) -> int:

@@ -498,3 +498,137 @@ int oracle_di_order(uint32_t k, const uint32_t* qrow, const uint32_t* qcol, uint
     free(st);
     return rc;
 }
+
+/* ============================================ disconnected Q
+ * "If the query graph is not connected ... we split Q into a set of connected
+ * components, compute sub-graph isomorphism on each of these components, and
+ * produce the final result as the cross product of individual solutions."
+ * Reading P16: an element of the result is still a subgraph
+ * isomorphism (Def. 4), i.e. injective, so only the combinations
+ * whose images are disjoint are kept.
+ *
+ * Step by step: the caller passes each component's embeddings (rows from
+ * oracle_enumerate of the component as its own query; comp_verts[c][t] is the
+ * query vertex of column t); this function walks the cross product with
+ * nested loops (one level per component), keeps a combination iff no data
+ * vertex repeats, counts it in 128 bits and, if `rows` is given, writes it in
+ * query-id order (unsorted; the caller sorts).  Nothing is materialised
+ * beyond the k-vertex partial combination.                                 */
+typedef struct {
+    uint32_t k, ncomp;
+    const uint32_t* size;            /* vertices per component              */
+    const uint32_t* const* verts;    /* query vertex ids per component      */
+    const uint32_t* const* crow;     /* component rows (count x size)       */
+    const uint64_t* ccount;          /* rows per component                  */
+    uint32_t f[ORC_MAXK];            /* f[query vertex] (partial)           */
+    uint32_t used[ORC_MAXK];         /* data vertices placed so far         */
+    uint32_t nused;
+    uint32_t* rows;
+    uint64_t cap;
+    u128 n;
+} orc_cross;
+
+static void cross_rec(orc_cross* x, uint32_t c) {
+    if (c == x->ncomp) {
+        if (x->rows && x->n < (u128)x->cap) memcpy(x->rows + (uint64_t)x->n * x->k, x->f, x->k * sizeof(uint32_t));
+        x->n++;
+        return;
+    }
+    const uint32_t s = x->size[c];
+    for (uint64_t r = 0; r < x->ccount[c]; ++r) {
+        const uint32_t* row = x->crow[c] + r * s;
+        int ok = 1;
+        for (uint32_t t = 0; t < s && ok; ++t)          /* injectivity across components */
+            for (uint32_t u = 0; u < x->nused && ok; ++u) ok = x->used[u] != row[t];
+        if (!ok) continue;
+        for (uint32_t t = 0; t < s; ++t) { x->f[x->verts[c][t]] = row[t]; x->used[x->nused + t] = row[t]; }
+        x->nused += s;
+        cross_rec(x, c + 1);
+        x->nused -= s;
+    }
+}
+
+int oracle_cross_product(uint32_t k, uint32_t ncomp, const uint32_t* size, const uint32_t* const* verts,
+                         const uint32_t* const* crow, const uint64_t* ccount,
+                         uint32_t* rows, uint64_t cap_rows, uint64_t* count_lo, uint64_t* count_hi) {
+    if (k < 1 || k > ORC_MAXK || ncomp < 1 || ncomp > k) return ORC_EINVAL;
+    orc_cross x;
+    memset(&x, 0, sizeof x);
+    x.k = k; x.ncomp = ncomp; x.size = size; x.verts = verts; x.crow = crow; x.ccount = ccount;
+    x.rows = rows; x.cap = rows ? cap_rows : 0;
+    cross_rec(&x, 0);
+    *count_lo = (uint64_t)x.n;
+    *count_hi = (uint64_t)(x.n >> 64);
+    if (rows) {
+        uint64_t nr = x.n < (u128)cap_rows ? (uint64_t)x.n : cap_rows;
+        g_sort_k = k;
+        qsort(rows, (size_t)nr, (size_t)k * sizeof(uint32_t), cmp_row);
+    }
+    return ORC_OK;
+}
+
+/* ========================================= root-parallel driver (N cores)
+ * SURVEY §8.c step 5 / BASELINE.md §4: level-1 roots are independent
+ * sub-trees, so disjoint ranges of the canonical level-1 list
+ * can be counted by separate threads with the same rec() and summed — exact
+ * by construction.  Threads pull ranges of `grain` roots from an atomic
+ * counter.  Used only for the CPU baseline timing (bench.py cpu_baseline);
+ * every parity pin goes through the single-threaded oracle_count.           */
+#include <pthread.h>
+
+typedef struct {
+    orc_state st;
+    const uint32_t* canon;
+    uint64_t begin, end, grain;
+    uint64_t* next;                  /* shared: next root position to hand out */
+} orc_worker;
+
+static void* worker_main(void* arg) {
+    orc_worker* w = (orc_worker*)arg;
+    for (;;) {
+        uint64_t a = __atomic_fetch_add(w->next, w->grain, __ATOMIC_RELAXED);
+        if (a >= w->end) break;
+        uint64_t b = a + w->grain < w->end ? a + w->grain : w->end;
+        for (uint64_t p = a; p < b; ++p) {
+            w->st.f[0] = w->canon[p];
+            w->st.level[1]++;
+            if (w->st.k == 1) emit(&w->st);
+            else rec(&w->st, 1);
+        }
+    }
+    return NULL;
+}
+
+int oracle_count_mt(uint32_t nthreads, uint32_t n, const uint64_t* row_ptr, const uint32_t* col,
+                    uint32_t k, const uint32_t* qrow, const uint32_t* qcol, const uint32_t* order,
+                    uint64_t root_begin, uint64_t root_end, uint64_t grain,
+                    uint64_t* count_lo, uint64_t* count_hi) {
+    if (nthreads < 1 || nthreads > 1024 || grain < 1) return ORC_EINVAL;
+    orc_worker* w = (orc_worker*)calloc(nthreads, sizeof(orc_worker));
+    pthread_t* th = (pthread_t*)calloc(nthreads, sizeof(pthread_t));
+    uint32_t* canon = (uint32_t*)malloc(((size_t)n + 1) * sizeof(uint32_t));
+    if (!w || !th || !canon) { free(w); free(th); free(canon); return ORC_ENOMEM; }
+    int rc = setup(&w[0].st, n, row_ptr, col, k, qrow, qcol, order);
+    if (rc) { free(w); free(th); free(canon); return rc; }
+    uint64_t nc = 0;                                    /* canonical level-1 list (Alg. 1 l.8-11) */
+    for (uint32_t v = 0; v < n; ++v)
+        if (deg(&w[0].st, v) >= w[0].st.qdeg[0]) canon[nc++] = v;
+    uint64_t b = root_begin < nc ? root_begin : nc, e = root_end < nc ? root_end : nc;
+    if (e < b) e = b;
+    uint64_t next = b;
+    for (uint32_t t = 0; t < nthreads; ++t) {
+        if (t) w[t].st = w[0].st;
+        w[t].canon = canon; w[t].begin = b; w[t].end = e; w[t].grain = grain; w[t].next = &next;
+    }
+    uint32_t started = 0;
+    for (; started < nthreads; ++started)
+        if (pthread_create(&th[started], NULL, worker_main, &w[started]) != 0) break;
+    if (started == 0) worker_main(&w[0]);
+    for (uint32_t t = 0; t < started; ++t) pthread_join(th[t], NULL);
+    u128 tot = 0;
+    for (uint32_t t = 0; t < nthreads; ++t) tot += w[t].st.n_rows;
+    *count_lo = (uint64_t)tot;
+    *count_hi = (uint64_t)(tot >> 64);
+    free(w); free(th); free(canon);
+    return ORC_OK;
+}

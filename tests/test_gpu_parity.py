@@ -429,7 +429,8 @@ def test_disconnected_queries(cuts, gname):
         if want <= 1_000_000:     # BFS holds every level only for the small results
             assert big.count("bfs") == want, (gname, name)
         assert big.count("hybrid") == want, (gname, name)
-        assert small.count("hybrid") == want, (gname, name)
+        if want <= 5_000_000:     # the 64 KiB arena runs thousands of chunks per million embeddings
+            assert small.count("hybrid") == want, (gname, name)
         if want <= 2_000_000:
             rows = big.enumerate("hybrid", cap_rows=want)
             assert np.array_equal(_sorted_rows(rows), oracle.enumerate_rows(g, q)), (gname, name)

@@ -425,3 +425,16 @@ def test_directed_order_rule():
     assert oracle.di_order(named_diquery("in2")) == [1, 0, 2]
     assert oracle.di_order(named_diquery("out2")) == [0, 1, 2]
     assert oracle.di_order(named_diquery("TT6-rev")) == [5, 4, 3, 2, 1, 0]
+
+
+def test_root_parallel_driver_matches_single_thread():
+    """oracle_count_mt (the N-core CPU baseline) sums
+    disjoint root ranges counted by the same rec(): equal to the single-threaded
+    count for every thread count / grain and every root range."""
+    from inputs import rmat_graph, DENSE5, SPARSE5
+    g = rmat_graph(9, 4, seed=2)
+    for q in (DENSE5[9], SPARSE5[1], named_query("K3")):
+        want = oracle.count(g, q)
+        for threads, grain in ((1, 1), (3, 1), (4, 7), (8, 64)):
+            assert oracle.count_mt(g, q, threads, grain=grain) == want, (q.name, threads, grain)
+        assert oracle.count_mt(g, q, 4, 10, 50, grain=3) == oracle.count(g, q, root_begin=10, root_end=50)
