@@ -36,7 +36,7 @@ extern "C" {
 #endif
 
 #define CUTS_MAX_K 8
-#define CUTS_ABI_VERSION 2
+#define CUTS_ABI_VERSION 3
 
 typedef struct cuts_ctx cuts_ctx;
 
@@ -49,7 +49,7 @@ typedef enum {
     CUTS_ETRUNC = -5,       /* enumeration found more rows than cap_rows                */
     CUTS_ESTATE = -6,       /* call out of order                                        */
     CUTS_EUNSUPPORTED = -7, /* k > 8                                                    */
-    CUTS_ECOMM = -8         /* reserved for the multi-GPU layer                         */
+    CUTS_ECOMM = -8         /* NCCL / donation transport failure (multi-GPU layer)      */
 } cuts_status;
 
 typedef enum {
@@ -83,13 +83,19 @@ typedef struct {
     double   ms_extend;                /* device time of extend/count kernels (if timing)   */
     double   ms_plan;                  /* device time of plan + scan kernels (if timing)    */
     uint64_t extend_launches;          /* launches timed in ms_extend                       */
-    uint64_t alg_bytes_extend;         /* algorithmic bytes of the extend kernels (SURVEY
-                                          §8.d model; only with CUTS_DEBUG_BYTES)           */
+    uint64_t alg_bytes_extend;         /* algorithmic bytes of the extend kernels, SURVEY §8.d
+                                          model kept FIXED: 4 d per backward list of every
+                                          entry + 4 per intersection survivor + children
+                                          written (only with CUTS_DEBUG_BYTES)              */
     uint64_t alg_bytes_plan;           /* algorithmic bytes of the plan kernels (ditto)     */
     uint64_t hubs;                     /* vertices with an adjacency bitmap (see below)     */
     uint64_t hub_threshold;            /* degree threshold used for the bitmaps             */
     uint64_t donations;                /* work donations made (cuts_set_donation)           */
     uint64_t donated_entries;          /* prefixes given away by those donations            */
+    uint64_t alg_bytes_extend_needed;  /* bytes the extend path's own algorithm needs (source
+                                          actually streamed: shortest list, ancestor range or
+                                          set-difference searches; + output) — beside the
+                                          frozen §8.d model in alg_bytes_extend              */
 } cuts_stats;
 
 /* debug / instrumentation flags for cuts_set_debug */
@@ -252,6 +258,37 @@ cuts_status cuts_set_donation(cuts_ctx* ctx, cuts_poll_fn poll, cuts_ship_fn shi
 cuts_status cuts_trie_decode(cuts_ctx* ctx, uint32_t nlevels, const uint64_t* sizes,
                              const uint32_t* const* d_ca, const uint32_t* const* d_pa,
                              uint32_t* d_out);
+
+/* ------------------------------------------------------------ multi-GPU
+ * Row e of the hot path (Alg. 3): one
+ * process per GPU, D replicated on every rank (Alg. 3 gives every rank Q and
+ * D), level-1 roots partitioned, counts summed with one NCCL
+ * all-reduce (the path's only collective).  NCCL is resolved at run time
+ * (dlopen of libnccl.so.2, normally the copy torch already loaded); the
+ * single-GPU path never needs it. */
+#define CUTS_DIST_UID_BYTES 128
+
+/* Write a fresh ncclUniqueId (CUTS_DIST_UID_BYTES bytes) to the HOST buffer
+ * out_128B — call on one rank and broadcast it (e.g. torch.distributed).
+ * CUTS_ECOMM if NCCL cannot be loaded. */
+cuts_status cuts_dist_unique_id(void* out_128B);
+
+/* Join ctx to a world of `world` ranks as `rank` (collective: every rank calls
+ * it with the same id).  nccl_uid_128B: HOST copy of the id from
+ * cuts_dist_unique_id (may be NULL only when world == 1: no communicator).
+ * peers: reserved for peer-mapped donation inboxes, must be NULL (donated
+ * prefixes travel through the caller's transport, see cuts_set_donation).
+ * Afterwards the default root partition of every query (set by
+ * cuts_set_query, overridable with cuts_set_root_slice) is this rank's
+ * cyclic slice p % world == rank of the shuffled level-1 list.
+ * CUTS_EINVAL on bad rank/world, CUTS_ECOMM if NCCL fails. */
+cuts_status cuts_set_dist(cuts_ctx* ctx, int rank, int world, const void* nccl_uid_128B, const void* peers);
+
+/* Collective exact sum over the ranks of a 128-bit count (lo, hi) -> (*out_lo,
+ * *out_hi), e.g. the per-rank results of cuts_count: four 32-bit limbs in u64
+ * words, one ncclAllReduce(ncclUint64, ncclSum) on ctx's stream.
+ * Without a communicator (world == 1) it copies.  Host-synchronous. */
+cuts_status cuts_allreduce_count(cuts_ctx* ctx, uint64_t lo, uint64_t hi, uint64_t* out_lo, uint64_t* out_hi);
 
 #ifdef __cplusplus
 }

@@ -19,13 +19,15 @@ STATUS_NAMES = {0: "CUTS_OK", -1: "CUTS_EINVAL", -2: "CUTS_ENOMEM", -3: "CUTS_EC
 CUTS_BFS, CUTS_HYBRID = 0, 1
 CUTS_DEBUG_TIMING, CUTS_DEBUG_BYTES = 1, 2
 MAX_K = 8
+DIST_UID_BYTES = 128
 
 # the symbols include/cuts.h declares (tests check the library exports all of them)
 EXPORTED = ["cuts_version", "cuts_create", "cuts_destroy", "cuts_last_error", "cuts_load_graph",
             "cuts_load_digraph", "cuts_set_query_directed",
             "cuts_set_query", "cuts_set_root_range", "cuts_set_root_slice", "cuts_level1_size", "cuts_count",
             "cuts_enumerate", "cuts_get_stats", "cuts_set_debug", "cuts_trie_decode", "cuts_set_hub_threshold",
-            "cuts_set_prefixes", "cuts_set_donation"]
+            "cuts_set_prefixes", "cuts_set_donation", "cuts_dist_unique_id", "cuts_set_dist",
+            "cuts_allreduce_count"]
 
 # callback types of cuts_set_donation
 POLL_FN = ctypes.CFUNCTYPE(ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64)
@@ -48,7 +50,7 @@ class cuts_stats(ctypes.Structure):
                 ("extend_launches", ctypes.c_uint64), ("alg_bytes_extend", ctypes.c_uint64),
                 ("alg_bytes_plan", ctypes.c_uint64), ("hubs", ctypes.c_uint64),
                 ("hub_threshold", ctypes.c_uint64), ("donations", ctypes.c_uint64),
-                ("donated_entries", ctypes.c_uint64)]
+                ("donated_entries", ctypes.c_uint64), ("alg_bytes_extend_needed", ctypes.c_uint64)]
 
 
 _lib = None
@@ -84,6 +86,9 @@ def load() -> ctypes.CDLL:
         "cuts_trie_decode": ([P, u32, u64p, ctypes.POINTER(P), ctypes.POINTER(P), P], i32),
         "cuts_set_prefixes": ([P, u32, u64, P], i32),
         "cuts_set_donation": ([P, POLL_FN, SHIP_FN, P], i32),
+        "cuts_dist_unique_id": ([P], i32),
+        "cuts_set_dist": ([P, i32, i32, P, P], i32),
+        "cuts_allreduce_count": ([P, u64, u64, u64p, u64p], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

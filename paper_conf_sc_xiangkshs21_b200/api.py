@@ -180,6 +180,11 @@ class Cuts:
             return self
         assert rows.dim() == 2 and rows.element_size() == 4 and rows.is_cuda
         rows = rows.contiguous()
+        # the rows may come from another stream (a recv, a copy): the library reads
+        # them on its own stream, so order it after everything queued so far
+        torch.cuda.current_stream(self.device).synchronize()
+        if rows.device != self.device:
+            raise ValueError("prefix rows must live on the context's device")
         self._prefixes = rows                   # borrowed by the library until the next run
         cnt, depth = rows.shape
         self._check(self.lib.cuts_set_prefixes(self.h, depth, cnt, rows.data_ptr() if cnt else None))
@@ -210,8 +215,13 @@ class Cuts:
                 if not count:
                     ship(int(depth), None)
                     return 0
-                view = torch.as_tensor(_DevRows(ptr, int(count), int(depth)), device=dev)
-                ship(int(depth), view.clone())
+                # clone on the library's stream and wait for it: once ship returns the
+                # library reuses that arena scratch for the next kernels on its stream
+                with torch.cuda.stream(self.stream):
+                    view = torch.as_tensor(_DevRows(ptr, int(count), int(depth)), device=dev)
+                    rows = view.clone()
+                self.stream.synchronize()
+                ship(int(depth), rows)
                 return 0
             except Exception:
                 import traceback
@@ -221,6 +231,34 @@ class Cuts:
         self._cb = (L.POLL_FN(_poll), L.SHIP_FN(_ship))
         self._check(self.lib.cuts_set_donation(self.h, self._cb[0], self._cb[1], None))
         return self
+
+    # ------------------------------------------------------------ multi-GPU
+    @staticmethod
+    def dist_unique_id() -> bytes:
+        """A fresh NCCL unique id (cuts_dist_unique_id): create on one rank, broadcast."""
+        lib = L.load()
+        buf = ctypes.create_string_buffer(L.DIST_UID_BYTES)
+        rc = lib.cuts_dist_unique_id(buf)
+        if rc != 0:
+            raise CutsError(rc, "cuts_dist_unique_id failed (NCCL not loadable)")
+        return buf.raw
+
+    def set_dist(self, rank: int, world: int, uid: bytes | None):
+        """cuts_set_dist: join a world (collective over the ranks when uid is given).
+        Afterwards every query defaults to this rank's cyclic level-1 slice."""
+        ub = None if uid is None else ctypes.create_string_buffer(bytes(uid), L.DIST_UID_BYTES)
+        self._check(self.lib.cuts_set_dist(self.h, int(rank), int(world), ub, None))
+        self.rank, self.world = int(rank), int(world)
+        return self
+
+    def allreduce_count(self, count: int) -> int:
+        """cuts_allreduce_count: exact 128-bit sum of `count` over the ranks (NCCL)."""
+        if count < 0 or count >= 1 << 128:
+            raise ValueError("count out of range")
+        lo, hi = ctypes.c_uint64(), ctypes.c_uint64()
+        self._check(self.lib.cuts_allreduce_count(self.h, count & (2**64 - 1), count >> 64,
+                                                  ctypes.byref(lo), ctypes.byref(hi)))
+        return int(lo.value) | (int(hi.value) << 64)
 
     def level1_size(self):
         """(canonical level-1 size, size inside the root range) for the current query."""
@@ -272,6 +310,7 @@ class Cuts:
             "extend_launches": s.extend_launches, "alg_bytes_extend": s.alg_bytes_extend,
             "alg_bytes_plan": s.alg_bytes_plan, "hubs": s.hubs, "hub_threshold": s.hub_threshold,
             "donations": s.donations, "donated_entries": s.donated_entries,
+            "alg_bytes_extend_needed": s.alg_bytes_extend_needed,
         }
 
     def trie_decode(self, ca_levels, pa_levels) -> torch.Tensor:

@@ -9,6 +9,8 @@
 // item offsets, scan temp).  HYBRID mode is a DFS over item-range chunks with
 // BFS inside each chunk; BFS mode stores each level whole.
 #include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>   // types and enum values only: the functions are resolved at run time (dlsym)
 #include <cub/device/device_scan.cuh>
 #include <cub/device/device_select.cuh>
 #include <thrust/iterator/counting_iterator.h>
@@ -92,12 +94,44 @@ struct cuts_ctx {
     uint32_t need_ord = 0;
     struct OrdState { const uint64_t* cpos; uint64_t w0; uint64_t ea; const uint2* lv; bool valid; };
     OrdState ord[kMaxK + 1] = {};
+    // multi-GPU (cuts_set_dist): rank / world and the NCCL communicator of the count reduction
+    int rank = 0, world = 1;
+    ncclComm_t comm = nullptr;
     uint64_t dfs_next[kMaxK + 1] = {};   // first entry of level d not yet planned
     uint64_t dfs_end[kMaxK + 1] = {};    // end of level d's entries still owned here
     bool dfs_on[kMaxK + 1] = {};
 };
 
 namespace {
+
+// NCCL through dlopen: the process normally has it loaded already (torch's
+// libnccl.so.2), so RTLD_NOLOAD reuses that copy; libcuts.so has no link-time
+// NCCL dependency and the single-GPU path never touches it.
+struct NcclApi {
+    decltype(&ncclGetUniqueId) get_unique_id = nullptr;
+    decltype(&ncclCommInitRank) init_rank = nullptr;
+    decltype(&ncclAllReduce) all_reduce = nullptr;
+    decltype(&ncclCommDestroy) destroy = nullptr;
+    decltype(&ncclGetErrorString) error_string = nullptr;
+    bool tried = false, ok = false;
+};
+
+NcclApi& nccl() {
+    static NcclApi api;
+    if (api.tried) return api;
+    api.tried = true;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return api;
+    api.get_unique_id = (decltype(api.get_unique_id))dlsym(h, "ncclGetUniqueId");
+    api.init_rank = (decltype(api.init_rank))dlsym(h, "ncclCommInitRank");
+    api.all_reduce = (decltype(api.all_reduce))dlsym(h, "ncclAllReduce");
+    api.destroy = (decltype(api.destroy))dlsym(h, "ncclCommDestroy");
+    api.error_string = (decltype(api.error_string))dlsym(h, "ncclGetErrorString");
+    api.ok = api.get_unique_id && api.init_rank && api.all_reduce && api.destroy && api.error_string;
+    return api;
+}
 
 cuts_status fail(cuts_ctx* c, cuts_status s, const char* fmt, ...) {
     char buf[512];
@@ -974,7 +1008,8 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     }
     if (k > 1) ctx->st.level_size[k] = ctx->st.count_lo;
     ctx->st.alg_bytes_plan = ctx->h_ctrl[kBytesPlan];
-    ctx->st.alg_bytes_extend = ctx->h_ctrl[kBytesExt];
+    ctx->st.alg_bytes_extend = ctx->h_ctrl[kBytesExt] + ctx->h_ctrl[kBytesOut];
+    ctx->st.alg_bytes_extend_needed = ctx->h_ctrl[kBytesNeed] + ctx->h_ctrl[kBytesOut];
     ctx->st.peak_arena_bytes = ctx->peak;
     ctx->st.hubs = ctx->nhubs;
     ctx->st.hub_threshold = ctx->hub_t_used;
@@ -1021,8 +1056,8 @@ cuts_status finish_query(cuts_ctx* ctx, const QPlan& qp, bool directed) {
     ctx->root_end = ~0ull;
     ctx->slice_begin = 0;
     ctx->slice_end = ~0ull;
-    ctx->part = 0;
-    ctx->nparts = 1;
+    ctx->part = (uint32_t)ctx->rank;      // after cuts_set_dist: this rank's cyclic slice
+    ctx->nparts = (uint32_t)ctx->world;   // of the shuffled level-1 list
     ctx->pre_j = 0;
     ctx->pre_count = 0;
     ctx->pre_rows = nullptr;
@@ -1062,6 +1097,7 @@ cuts_status cuts_create(cuts_ctx** out, const cuts_opts* o) {
 
 void cuts_destroy(cuts_ctx* ctx) {
     if (!ctx) return;
+    if (ctx->comm && nccl().ok) nccl().destroy(ctx->comm);
     for (auto e : ctx->ev_pool) cudaEventDestroy(e);
     if (ctx->h_ctrl) cudaFreeHost(ctx->h_ctrl);
     delete ctx;
@@ -1301,6 +1337,72 @@ cuts_status cuts_trie_decode(cuts_ctx* ctx, uint32_t nlevels, const uint64_t* si
     }
     TRY(read_ctrl(ctx));
     if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_EINVAL, "parent index out of range");
+    return CUTS_OK;
+}
+
+cuts_status cuts_dist_unique_id(void* out_128B) {
+    if (!out_128B) return CUTS_EINVAL;
+    NcclApi& api = nccl();
+    if (!api.ok) return CUTS_ECOMM;
+    ncclUniqueId id;
+    if (api.get_unique_id(&id) != ncclSuccess) return CUTS_ECOMM;
+    static_assert(sizeof(ncclUniqueId) == CUTS_DIST_UID_BYTES, "ncclUniqueId size");
+    memcpy(out_128B, &id, sizeof id);
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_dist(cuts_ctx* ctx, int rank, int world, const void* nccl_uid_128B, const void* peers) {
+    if (!ctx) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (world < 1 || rank < 0 || rank >= world) return fail(ctx, CUTS_EINVAL, "bad rank %d / world %d", rank, world);
+    if (peers) return fail(ctx, CUTS_EINVAL, "peers is reserved and must be NULL");
+    if (world > 1 && !nccl_uid_128B) return fail(ctx, CUTS_EINVAL, "world %d needs an NCCL unique id", world);
+    CK(cudaSetDevice(ctx->device));
+    NcclApi& api = nccl();
+    if (ctx->comm) {
+        if (api.ok) api.destroy(ctx->comm);
+        ctx->comm = nullptr;
+    }
+    if (nccl_uid_128B) {   // world 1 with an id still builds a (trivial) communicator
+        if (!api.ok) return fail(ctx, CUTS_ECOMM, "libnccl.so.2 not found (dlopen)");
+        ncclUniqueId id;
+        memcpy(&id, nccl_uid_128B, sizeof id);
+        const ncclResult_t r = api.init_rank(&ctx->comm, world, id, rank);
+        if (r != ncclSuccess) {
+            ctx->comm = nullptr;
+            return fail(ctx, CUTS_ECOMM, "ncclCommInitRank(world %d, rank %d): %s", world, rank, api.error_string(r));
+        }
+    }
+    ctx->rank = rank;
+    ctx->world = world;
+    ctx->part = (uint32_t)rank;
+    ctx->nparts = (uint32_t)world;
+    return CUTS_OK;
+}
+
+cuts_status cuts_allreduce_count(cuts_ctx* ctx, uint64_t lo, uint64_t hi, uint64_t* out_lo, uint64_t* out_hi) {
+    if (!ctx || !out_lo || !out_hi) return CUTS_EINVAL;
+    ctx->err.clear();
+    if (ctx->world == 1 && !ctx->comm) {
+        *out_lo = lo;
+        *out_hi = hi;
+        return CUTS_OK;
+    }
+    if (!ctx->comm) return fail(ctx, CUTS_ESTATE, "cuts_set_dist with an NCCL id must precede cuts_allreduce_count");
+    CK(cudaSetDevice(ctx->device));
+    // four 32-bit limbs in u64 words: each limb sum is <= world * (2^32 - 1), no overflow
+    unsigned long long* h = ctx->h_ctrl + kCtrlWords + 8;
+    unsigned long long* d = ctx->ctrl + kDistLimbs;
+    h[0] = lo & 0xffffffffull; h[1] = lo >> 32; h[2] = hi & 0xffffffffull; h[3] = hi >> 32;
+    CK(cudaMemcpyAsync(d, h, 4 * sizeof(unsigned long long), cudaMemcpyHostToDevice, ctx->stream));
+    const ncclResult_t r = nccl().all_reduce(d, d, 4, ncclUint64, ncclSum, ctx->comm, ctx->stream);
+    if (r != ncclSuccess) return fail(ctx, CUTS_ECOMM, "ncclAllReduce: %s", nccl().error_string(r));
+    CK(cudaMemcpyAsync(h, d, 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    unsigned __int128 t = (unsigned __int128)h[0] + ((unsigned __int128)h[1] << 32) + ((unsigned __int128)h[2] << 64) +
+                          ((unsigned __int128)h[3] << 96);
+    *out_lo = (uint64_t)t;
+    *out_hi = (uint64_t)(t >> 64);
     return CUTS_OK;
 }
 

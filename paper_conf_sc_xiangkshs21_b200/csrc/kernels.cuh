@@ -97,8 +97,14 @@ constexpr uint32_t kBmFlag = 0x80000000u;   // list-slot length flag: probe a bi
 enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 
 // control block (u64 words in the arena)
+// algorithmic bytes (CUTS_DEBUG_BYTES; SURVEY §8.d model, frozen): kBytesPlan = entry + path
+// hops + list bounds; kBytesExt = every backward list read once (4 d per list, whatever
+// source the kernel streams) + 4 per intersection survivor; kBytesOut = children written;
+// kBytesNeed = the source bytes this kernel's algorithm actually needs (shortest list,
+// ancestor range, or the set-difference searches), reported beside the model
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
-            kEnumCursor = 6, kNumSel = 7, kWork = 8, kFind = 24, kCtrlWords = 64 };
+            kEnumCursor = 6, kNumSel = 7, kWork = 8, kBytesOut = 9, kBytesNeed = 10, kFind = 24,
+            kDistLimbs = 56, kCtrlWords = 64 };
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
     if (v == 0) return;
@@ -274,7 +280,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
     const uint32_t bw = q.bw[J];
     const uint32_t bwi = q.bwi[J];
     constexpr int J2 = D ? 2 * J : J;   // list slots: [0, J) children of path[p], [J, 2J) parents (directed)
-    unsigned long long bytes_plan = 0, bytes_ext = 0;
+    unsigned long long bytes_plan = 0, bytes_ext = 0, bytes_need = 0;
     for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e <= W; e += gridDim.x * blockDim.x) {
         if (e == W) { ub[W] = 0; continue; }
         uint32_t path[J];
@@ -370,21 +376,24 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         for (int p = 0; p < J; ++p) path_s[(size_t)p * W + e] = path[p];
         if (count_bytes) {   // 8 (entry) + 8(J-1) (hops) + 16 per list bound
             bytes_plan += 8ull + 8ull * (J - 1) + 16ull * __popc(need);
-            if (trie) {          // the ancestor range (8 B entries) + the lists not covered by it
-                bytes_ext += 8ull * trie_len + 4ull * rest_sum;
+            bytes_ext += 4ull * lists;                   // the model: every backward list read once
+            if (trie) {          // needed: the ancestor range (8 B entries) + the lists not covered by it
+                bytes_need += 8ull * trie_len + 4ull * rest_sum;
             } else if (fast_last<J>(q, need, g.dn ? 0u : 1u)) {   // J binary searches in the list
-                bytes_ext += 4ull * J * (32 - __clz(best_d));
+                bytes_need += 4ull * J * (32 - __clz(best_d));
             } else {
-                bytes_ext += 4ull * lists;               // every backward list read once
+                bytes_need += 4ull * lists;
             }
         }
     }
     if (count_bytes) {
         bytes_plan = warp_sum(bytes_plan);
         bytes_ext = warp_sum(bytes_ext);
+        bytes_need = warp_sum(bytes_need);
         if ((threadIdx.x & 31) == 0) {
             atomicAdd(ctrl + kBytesPlan, bytes_plan);
             atomicAdd(ctrl + kBytesExt, bytes_ext);
+            atomicAdd(ctrl + kBytesNeed, bytes_need);
         }
     }
 }
@@ -448,7 +457,7 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
     // undirected: a candidate from a list has deg >= 1, so qdeg <= 1 needs no check;
     // directed: a child may have out-degree 0
     const uint32_t qmin = g.dn ? 0u : 1u;
-    unsigned long long my_count = 0, bytes = 0;
+    unsigned long long my_count = 0, bytes = 0, obytes = 0;   // bytes: 4 per survivor; obytes: output
     unsigned int* work = (unsigned int*)(ctrl + kWork);
     const unsigned long long wbytes = M == kCount ? 0ull : (M == kEnum ? 4ull * q.k : 8ull);
 
@@ -545,6 +554,7 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                 // |list[ilo, ihi) \ path|: lane vl < J looks for path[vl] (a distinct vertex)
                 if (has) {
                     unsigned long long c = vl == 0 ? (unsigned long long)(ihi - ilo) : 0ull;
+                    if (count_bytes && vl == 0) bytes += 4ull * (ihi - ilo);   // model: every element survives
                     if (vl < J && ihi > ilo) {
                         uint32_t x = path[0];
 #pragma unroll
@@ -557,7 +567,6 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                             len -= half;
                         }
                         if (__ldg(b0) == x) c -= 1ull;    // u64 wrap: the warp sum is exact
-                        if (count_bytes) bytes += 4ull * (32 - __clz(ihi - ilo));
                     }
                     my_count += c;
                     ecnt += c;
@@ -586,8 +595,10 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                         k0 = k0 && d0 >= qd;
                         k1 = k1 && d1 >= qd;
                     }
-                    if (count_bytes)
-                        bytes += (a0 ? 4ull : 0ull) + (a1 ? 4ull : 0ull) + (k0 ? wbytes : 0ull) + (k1 ? wbytes : 0ull);
+                    if (count_bytes) {
+                        bytes += (a0 ? 4ull : 0ull) + (a1 ? 4ull : 0ull);
+                        obytes += (k0 ? wbytes : 0ull) + (k1 ? wbytes : 0ull);
+                    }
                     emit(k0, c0);
                     if (it + 1 < nit_max) emit(k1, c1);
                 }
@@ -638,7 +649,10 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                         if (pv) { lb[x] += mpos; ln[x] -= mpos; }
                     }
                 }
-                if (count_bytes) bytes += (inter ? 4ull : 0ull) + (inter && ok ? wbytes : 0ull);
+                if (count_bytes) {
+                    bytes += inter ? 4ull : 0ull;
+                    obytes += inter && ok ? wbytes : 0ull;
+                }
                 ok = ok && inter;
                 emit(ok, c);
             }
@@ -656,7 +670,11 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
     }
     if (count_bytes) {
         bytes = warp_sum(bytes);
-        if (lane == 0) atomicAdd(ctrl + kBytesExt, bytes);
+        obytes = warp_sum(obytes);
+        if (lane == 0) {
+            atomicAdd(ctrl + kBytesExt, bytes);
+            atomicAdd(ctrl + kBytesOut, obytes);
+        }
     }
 }
 

@@ -42,10 +42,14 @@ def n_chunks(level1: int, chunk_size: int) -> int:
     return (level1 + chunk_size - 1) // chunk_size if chunk_size > 0 else 0
 
 
-def allreduce_count(count: int, group=None, device=None) -> int:
-    """Exact sum over ranks of a non-negative integer < 2^128 (limbs of 32 bits in int64)."""
+def allreduce_count(count: int, group=None, device=None, ctx=None) -> int:
+    """Exact sum over ranks of a non-negative integer < 2^128.  With a context that
+    joined a world (``Cuts.set_dist``) the library's own NCCL all-reduce does it
+    (cuts_allreduce_count); otherwise 32-bit limbs in int64 over torch.distributed."""
     if count < 0 or count >= 1 << (_LIMB * _NLIMB):
         raise ValueError("count out of range")
+    if ctx is not None and getattr(ctx, "world", 1) > 1:
+        return ctx.allreduce_count(count)
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size(group) == 1:
         return count
     limbs = [(count >> (_LIMB * i)) & _MASK for i in range(_NLIMB)]
@@ -249,7 +253,7 @@ class CutsEngine:
         return c
 
     def count_prefixes(self, rows) -> int:
-        rows = rows.to(self.ctx.device)
+        rows = rows.to(self.ctx.device)      # set_prefixes orders the library's stream after this copy
         self.ctx.set_prefixes(rows)
         try:
             c = self.ctx.count(self.mode)

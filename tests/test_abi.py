@@ -30,7 +30,7 @@ def lib():
 def test_header_declares_the_boundary():
     names = _declared()
     for must in ["cuts_create", "cuts_destroy", "cuts_last_error", "cuts_load_graph", "cuts_set_query",
-                 "cuts_count", "cuts_enumerate", "cuts_set_root_range", "cuts_get_stats"]:
+                 "cuts_count", "cuts_enumerate", "cuts_set_root_range", "cuts_set_dist", "cuts_get_stats"]:
         assert must in names
 
 
@@ -43,7 +43,7 @@ def test_library_exports_every_declared_symbol(lib):
 
 def test_version_and_null_args(lib):
     lib.cuts_version.restype = ctypes.c_int
-    assert lib.cuts_version() == 2
+    assert lib.cuts_version() == 3
     lib.cuts_create.restype = ctypes.c_int
     lib.cuts_create.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
     assert lib.cuts_create(None, None) == -1                  # CUTS_EINVAL, no CUDA call
