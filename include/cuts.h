@@ -96,6 +96,9 @@ typedef struct {
                                           actually streamed: shortest list, ancestor range or
                                           set-difference searches; + output) — beside the
                                           frozen §8.d model in alg_bytes_extend              */
+    uint64_t free_identity;            /* disconnected Q: 1 if the component roots streamed the
+                                          identity list [0, n) with an in-kernel degree
+                                          filter (the filtered lists did not fit the arena)  */
 } cuts_stats;
 
 /* debug / instrumentation flags for cuts_set_debug */
@@ -110,6 +113,17 @@ typedef struct {
 #define CUTS_DEBUG_NO_FAST_COUNT 32u /* ablation: stream the list at a single-list,
                                   degree-free last level of cuts_count instead of counting
                                   |list| - |path found in list| by binary search            */
+#define CUTS_DEBUG_PRELOAD_COUNT 64u /* test hook: cuts_count starts its 128-bit counter at
+                                  2^64 - 2^20 instead of 0 (exercises the carry into the
+                                  high word and CUTS_EOVERFLOW; the result is offset)      */
+#define CUTS_DEBUG_BINNED 128u /* ablation (NEXT-2): the last level groups its entries into
+                                  bins by work and runs each bin with its own virtual-warp
+                                  width instead of one bin sized by the average
+                                  (the paper's choice)                          */
+#define CUTS_DEBUG_SV 256u     /* ablation (NEXT-2): scatter-vector intersection (Alg. 2
+                                  l.7-17) with a u8 sv[n] per warp in the arena,
+                                  CSR lists only (no hub bitmaps, no ancestor source, no
+                                  set-difference count); undirected; count/write modes      */
 
 /* Create a context bound to opts->device / opts->stream / opts->arena.
  * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */

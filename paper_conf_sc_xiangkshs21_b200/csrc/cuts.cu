@@ -34,6 +34,7 @@ constexpr uint64_t kAlign = 256;
 constexpr uint64_t kCtrlBytes = 4096;
 constexpr uint64_t kMaxWindow = 1ull << 24;      // entries per plan window
 constexpr uint64_t kMaxLevel = 0xFFFFFFFFull;    // u32 parent indices
+constexpr uint64_t kPreloadCount = 0xFFFFFFFFFFF00000ull;   // CUTS_DEBUG_PRELOAD_COUNT: 2^64 - 2^20
 
 inline uint64_t align_up(uint64_t x) { return (x + kAlign - 1) & ~(kAlign - 1); }
 
@@ -64,6 +65,12 @@ struct cuts_ctx {
     uint64_t nhubs = 0, hub_t_used = 0;
     uint32_t hub_t = 0;                    // requested threshold (0 auto, UINT32_MAX off)
     uint64_t base_off = 0;                 // first free byte after ctrl + deg + bitmaps
+    // canonical level-1 list of the current query (Alg. 1 l.8-11), built once per
+    // (graph, query) right after base_off and reused by every count / root chunk
+    bool canon_valid = false;
+    uint32_t* canon = nullptr;
+    uint64_t canon_n = 0;
+    uint64_t run_off = 0;                  // first free byte after the canonical list
     // query
     bool has_query = false;
     bool q_directed = false;
@@ -94,6 +101,9 @@ struct cuts_ctx {
     uint32_t need_ord = 0;
     struct OrdState { const uint64_t* cpos; uint64_t w0; uint64_t ea; const uint2* lv; bool valid; };
     OrdState ord[kMaxK + 1] = {};
+    // CUTS_DEBUG_SV: per-warp u8 scatter vectors of n entries (zeroed; kernels leave them clean)
+    uint8_t* sv = nullptr;
+    uint64_t sv_warps = 0;
     // multi-GPU (cuts_set_dist): rank / world and the NCCL communicator of the count reduction
     int rank = 0, world = 1;
     ncclComm_t comm = nullptr;
@@ -363,6 +373,9 @@ struct Window {
     void* cub_tmp;
     size_t cub_bytes;
     uint64_t total;
+    const uint32_t* elist = nullptr;     // binned launch: explicit entry list (one bin)
+    uint32_t elist_n = 0;
+    int force_g = 0;                     // binned launch: that bin's virtual-warp width
 };
 
 template <int J>
@@ -407,15 +420,19 @@ void launch_extend_g(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0
                                                                    out_level, out_rows, cap, ctx->ctrl,
                                                                    (ctx->debug & CUTS_DEBUG_BYTES) && !w.ord_cnt ? 1 : 0, batch,
                                                                    w.ru.a ? ctx->q.qdeg[w.ru.a] : 0u,
-                                                                   w.ru.lv, w.ord_cnt, w.ord_pos, w.ord_ea);
+                                                                   w.ru.lv, w.ord_cnt, w.ord_pos, w.ord_ea,
+                                                                   w.elist, w.elist_n);
 }
 
 template <int J, int NL, int M>
 void launch_extend_nl(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
                       uint2* out_level, uint32_t* out_rows, uint64_t cap) {
-    // virtual-warp width from the average candidate-list length
+    // virtual-warp width from the average candidate-list length, or the bin's
     const double avg = (double)w.total / (double)std::max<uint32_t>(w.W, 1);
-    if (avg >= 96) launch_extend_g<J, NL, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    if (w.force_g == 32) launch_extend_g<J, NL, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else if (w.force_g == 16) launch_extend_g<J, NL, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else if (w.force_g == 8) launch_extend_g<J, NL, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else if (avg >= 96) launch_extend_g<J, NL, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
     else if (avg >= 24) launch_extend_g<J, NL, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
     else launch_extend_g<J, NL, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
 }
@@ -448,6 +465,45 @@ void launch_extend_m(cuts_ctx* ctx, int J, const Graph& g, const Window& w, uint
         case 6: launch_extend_t<6, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
         case 7: launch_extend_t<7, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
     }
+}
+
+template <int J, int NL, int M>
+void launch_extend_sv_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1, uint2* out,
+                        uint64_t cap) {
+    k_extend_sv<J, NL, M><<<(unsigned)(ctx->sv_warps / 8), 256, 0, ctx->stream>>>(
+        g, ctx->q, w.w0, w.W, w.path, w.src, w.offs, w.lst_off, w.lst_len, t0, t1, out, cap, ctx->ctrl, ctx->sv,
+        (uint64_t)ctx->n);
+}
+
+template <int J, int M>
+void launch_extend_sv_j(cuts_ctx* ctx, int nl, const Graph& g, const Window& w, uint64_t t0, uint64_t t1, uint2* out,
+                        uint64_t cap) {
+    switch (nl) {
+        case 1: if constexpr (J > 1) launch_extend_sv_t<J, (J > 1 ? 1 : 1), M>(ctx, g, w, t0, t1, out, cap); break;
+        case 2: if constexpr (J > 2) launch_extend_sv_t<J, (J > 2 ? 2 : 1), M>(ctx, g, w, t0, t1, out, cap); break;
+        case 3: if constexpr (J > 3) launch_extend_sv_t<J, (J > 3 ? 3 : 1), M>(ctx, g, w, t0, t1, out, cap); break;
+        case 4: if constexpr (J > 4) launch_extend_sv_t<J, (J > 4 ? 4 : 1), M>(ctx, g, w, t0, t1, out, cap); break;
+        case 5: if constexpr (J > 5) launch_extend_sv_t<J, (J > 5 ? 5 : 1), M>(ctx, g, w, t0, t1, out, cap); break;
+        case 6: if constexpr (J > 6) launch_extend_sv_t<J, (J > 6 ? 6 : 1), M>(ctx, g, w, t0, t1, out, cap); break;
+    }
+}
+
+// SV ablation launch; false if this level has no list to intersect (NL = 0)
+template <int M>
+bool launch_extend_sv(cuts_ctx* ctx, int J, const Graph& g, const Window& w, uint64_t t0, uint64_t t1, uint2* out,
+                      uint64_t cap) {
+    const int nl = __builtin_popcount(ctx->q.bw[J]) - 1;
+    if (nl < 1) return false;
+    switch (J) {
+        case 2: launch_extend_sv_j<2, M>(ctx, nl, g, w, t0, t1, out, cap); break;
+        case 3: launch_extend_sv_j<3, M>(ctx, nl, g, w, t0, t1, out, cap); break;
+        case 4: launch_extend_sv_j<4, M>(ctx, nl, g, w, t0, t1, out, cap); break;
+        case 5: launch_extend_sv_j<5, M>(ctx, nl, g, w, t0, t1, out, cap); break;
+        case 6: launch_extend_sv_j<6, M>(ctx, nl, g, w, t0, t1, out, cap); break;
+        case 7: launch_extend_sv_j<7, M>(ctx, nl, g, w, t0, t1, out, cap); break;
+        default: return false;
+    }
+    return true;
 }
 
 // ---- the level pipeline ----------------------------------------------------
@@ -500,7 +556,11 @@ cuts_status extend_range(cuts_ctx* ctx, Run& r, int J, const Window& w, uint64_t
     int e0 = -1;
     CK(cudaMemsetAsync(ctx->ctrl + kWork, 0, sizeof(unsigned long long), ctx->stream));
     if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
-    if (mode == kWrite) launch_extend_m<kWrite>(ctx, J, r.g, w, t0, t1, out, nullptr, cap);
+    const bool sv = ctx->sv && mode != kEnum && !w.ord_cnt && !w.ord_pos && !w.elist &&
+                    (mode == kWrite ? launch_extend_sv<kWrite>(ctx, J, r.g, w, t0, t1, out, cap)
+                                    : launch_extend_sv<kCount>(ctx, J, r.g, w, t0, t1, nullptr, 0));
+    if (sv) {
+    } else if (mode == kWrite) launch_extend_m<kWrite>(ctx, J, r.g, w, t0, t1, out, nullptr, cap);
     else if (mode == kCount) launch_extend_m<kCount>(ctx, J, r.g, w, t0, t1, nullptr, nullptr, 0);
     else launch_extend_m<kEnum>(ctx, J, r.g, w, t0, t1, nullptr, r.rows, r.cap_rows);
     CK(cudaGetLastError());
@@ -511,6 +571,37 @@ cuts_status extend_range(cuts_ctx* ctx, Run& r, int J, const Window& w, uint64_t
     }
     ctx->st.chunks++;
     ctx->st.launches++;
+    return CUTS_OK;
+}
+
+// last level over the whole window: one launch with the window's single-bin
+// virtual warp (the paper's choice), or with CUTS_DEBUG_BINNED one
+// launch per non-empty bin of entries grouped by work
+cuts_status extend_last(cuts_ctx* ctx, Run& r, int J, const Window& w, int mode) {
+    if (!(ctx->debug & CUTS_DEBUG_BINNED) || w.total == 0)
+        return extend_range(ctx, r, J, w, 0, w.total, mode, nullptr, 0);
+    const uint64_t top_save = ctx->top;
+    uint64_t off;
+    TRY(alloc_top(ctx, 3ull * w.W * 4, &off));
+    uint32_t* bins = (uint32_t*)(ctx->arena + off);
+    CK(cudaMemsetAsync(ctx->ctrl + kBins, 0, 3 * sizeof(unsigned long long), ctx->stream));
+    const unsigned grid = (unsigned)std::min<uint64_t>((w.W + 255) / 256, (uint64_t)ctx->num_sms * 8);
+    k_bin<<<grid, 256, 0, ctx->stream>>>(w.ub, w.W, bins, ctx->ctrl + kBins);
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(ctx->h_ctrl + kBins, ctx->ctrl + kBins, 3 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->st.launches++;
+    static const int kG[3] = {8, 16, 32};
+    for (int b = 0; b < 3; ++b) {
+        const uint64_t nb = ctx->h_ctrl[kBins + b];
+        if (!nb) continue;
+        Window wb = w;
+        wb.elist = bins + (size_t)b * w.W;
+        wb.elist_n = (uint32_t)nb;
+        wb.force_g = kG[b];
+        TRY(extend_range(ctx, r, J, wb, 0, w.total, mode, nullptr, 0));
+    }
+    ctx->top = top_save;
     return CUTS_OK;
 }
 
@@ -593,7 +684,7 @@ cuts_status maybe_donate(cuts_ctx* ctx, Run& r) {
 
 // HYBRID: process entries [0, N) of level J stored at r.t.lv[J] (DFS over chunks)
 inline bool reuse_on(const cuts_ctx* ctx, const Run& r) {
-    return r.mode == CUTS_HYBRID && !(ctx->debug & CUTS_DEBUG_NO_REUSE);
+    return r.mode == CUTS_HYBRID && !(ctx->debug & (CUTS_DEBUG_NO_REUSE | CUTS_DEBUG_SV));
 }
 
 // level J+1's chunk share of the free space: deeper stored levels (J+2 .. k-1)
@@ -716,7 +807,7 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
         TRY(alloc_window(ctx, J, w.W, &w));
         TRY(plan_window(ctx, r, J, w));
         if (last) {
-            TRY(extend_range(ctx, r, J, w, 0, w.total, r.enumerate ? kEnum : kCount, nullptr, 0));
+            TRY(extend_last(ctx, r, J, w, r.enumerate ? kEnum : kCount));
         } else if (ordered) {
             TRY(hybrid_ordered(ctx, r, J, w));
         } else {
@@ -752,7 +843,8 @@ cuts_status bfs_levels(cuts_ctx* ctx, Run& r, int J0, uint64_t N1) {
             w.w0 = w0;
             w.W = (uint32_t)std::min<uint64_t>(W, N - w0);
             TRY(plan_window(ctx, r, J, w));
-            TRY(extend_range(ctx, r, J, w, 0, w.total, last ? (r.enumerate ? kEnum : kCount) : kWrite, out, cap));
+            if (last) TRY(extend_last(ctx, r, J, w, r.enumerate ? kEnum : kCount));
+            else TRY(extend_range(ctx, r, J, w, 0, w.total, kWrite, out, cap));
             if (!last && w0 + W < N) {     // stop at the first window that overflows the level
                 CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
                 CK(cudaStreamSynchronize(ctx->stream));
@@ -830,11 +922,15 @@ cuts_status build_hubs(cuts_ctx* ctx) {
     return CUTS_OK;
 }
 
-// level 1: canonical list -> root range -> shuffle -> slice (P:938-942, P:916-922, P:1277-1279)
-cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
-    const uint64_t top_save = ctx->top;
+// canonical level-1 list {u : deg(u) >= deg_Q(S[0])} in ascending id (CUB select
+// over a counting iterator), cached per (graph, query): every root chunk of the
+// multi-GPU queue reuses it instead of re-running the O(n) select
+cuts_status ensure_canonical(cuts_ctx* ctx) {
+    if (ctx->canon_valid) return CUTS_OK;
+    ctx->bot = ctx->base_off;
+    ctx->top = ctx->arena_bytes & ~(kAlign - 1);
     uint64_t off_canon, off_tmp;
-    TRY(alloc_top(ctx, (uint64_t)ctx->n * 4 + 4, &off_canon));
+    TRY(alloc_bot(ctx, (uint64_t)ctx->n * 4 + 4, &off_canon));
     uint32_t* canon = (uint32_t*)(ctx->arena + off_canon);
     DegAtLeast pred{ctx->deg, ctx->q.qdeg[0], ctx->directed ? ctx->n : 0u, ctx->q.qdin[0]};
     thrust::counting_iterator<uint32_t> it(0);
@@ -844,7 +940,17 @@ cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
     TRY(alloc_top(ctx, tmp_bytes, &off_tmp));
     CK(cub::DeviceSelect::If(ctx->arena + off_tmp, tmp_bytes, it, canon, d_num, (int64_t)ctx->n, pred, ctx->stream));
     TRY(read_ctrl(ctx));
-    const uint64_t ncanon = ctx->h_ctrl[kNumSel];
+    ctx->canon = canon;
+    ctx->canon_n = ctx->h_ctrl[kNumSel];
+    ctx->run_off = align_up(off_canon + ctx->canon_n * 4 + 4);
+    ctx->canon_valid = true;
+    return CUTS_OK;
+}
+
+// level 1: canonical list -> root range -> shuffle -> slice (P:938-942, P:916-922, P:1277-1279)
+cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
+    const uint32_t* canon = ctx->canon;
+    const uint64_t ncanon = ctx->canon_n;
     ctx->st.level1_canonical = ncanon;
     uint64_t rb = std::min(ctx->root_begin, ncanon), re = std::min(ctx->root_end, ncanon);
     if (re < rb) re = rb;
@@ -880,8 +986,6 @@ cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
         CK(cudaGetLastError());
         ctx->st.launches++;
     }
-    ctx->st.launches += 2;
-    ctx->top = top_save;
     r.t.lv[1] = L1;
     *n1 = cnt;
     return CUTS_OK;
@@ -892,10 +996,21 @@ cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
 // on the bottom stack (the extend kernel reads it like a CSR source list)
 cuts_status build_free_lists(cuts_ctx* ctx, Run& r) {
     r.g.fre = (const uint32_t*)ctx->arena;
+    int roots = 0;
+    for (uint32_t J = 1; J < ctx->q.k; ++J) roots += (ctx->q.bw[J] | ctx->q.bwi[J]) ? 0 : 1;
+    // the lists take n u32 each: when they would crowd the trie (more than 1/8 of the
+    // free arena), a component root streams the identity list [0, n) instead and the
+    // extend kernel applies its degree filter (same candidates, no memory)
+    const bool identity = roots && (uint64_t)roots * ((uint64_t)ctx->n * 4 + 4 + kAlign) > free_bytes(ctx) / 8;
     for (uint32_t J = 1; J < ctx->q.k; ++J) {
         ctx->q.foff[J] = 0;
         ctx->q.flen[J] = 0;
         if (ctx->q.bw[J] | ctx->q.bwi[J]) continue;
+        if (identity) {
+            ctx->q.foff[J] = kIdSrc;
+            ctx->q.flen[J] = ctx->n;
+            continue;
+        }
         uint64_t off_list;
         TRY(alloc_bot(ctx, (uint64_t)ctx->n * 4 + 4, &off_list));
         const uint64_t top_save = ctx->top;
@@ -914,6 +1029,7 @@ cuts_status build_free_lists(cuts_ctx* ctx, Run& r) {
         ctx->q.flen[J] = (uint32_t)ctx->h_ctrl[kNumSel];
         ctx->st.launches += 2;
     }
+    ctx->st.free_identity = identity ? 1 : 0;
     return CUTS_OK;
 }
 
@@ -949,10 +1065,16 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     ctx->ev_used = 0;
     ctx->ev_ext.clear();
     ctx->ev_plan.clear();
-    ctx->bot = ctx->base_off;
+    if (!ctx->pre_j) TRY(ensure_canonical(ctx));
+    ctx->bot = ctx->canon_valid ? ctx->run_off : ctx->base_off;
     ctx->top = ctx->arena_bytes & ~(kAlign - 1);
     ctx->peak = ctx->bot;
     CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
+    if (ctx->debug & CUTS_DEBUG_PRELOAD_COUNT) {   // test hook: the 128-bit carry and CUTS_EOVERFLOW
+        ctx->h_ctrl[kCtrlWords + 16] = kPreloadCount;
+        CK(cudaMemcpyAsync(ctx->ctrl + kCountLo, ctx->h_ctrl + kCtrlWords + 16, 8, cudaMemcpyHostToDevice, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+    }
 
     Run r{};
     r.mode = mode;
@@ -965,7 +1087,21 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words, ctx->colx};
     r.g.dn = ctx->directed ? ctx->n : 0u;
     ctx->q.src_first = (ctx->debug & CUTS_DEBUG_FIRST_SOURCE) ? 1u : 0u;
-    ctx->q.count_fast = (!enumerate && !(ctx->debug & CUTS_DEBUG_NO_FAST_COUNT)) ? 1u : 0u;
+    ctx->q.count_fast = (!enumerate && !(ctx->debug & (CUTS_DEBUG_NO_FAST_COUNT | CUTS_DEBUG_SV))) ? 1u : 0u;
+    ctx->sv = nullptr;
+    ctx->sv_warps = 0;
+    if (ctx->debug & CUTS_DEBUG_SV) {   // ablation: per-warp scatter vectors, CSR lists only
+        if (ctx->directed) return fail(ctx, CUTS_EUNSUPPORTED, "CUTS_DEBUG_SV is undirected only");
+        r.g.hub = nullptr;
+        uint64_t warps = (uint64_t)ctx->num_sms * 16;
+        const uint64_t room = free_bytes(ctx) / 4;
+        while (warps > 8 && warps * ctx->n > room) warps /= 2;
+        uint64_t off;
+        TRY(alloc_bot(ctx, warps * ctx->n + 16, &off));
+        ctx->sv = (uint8_t*)(ctx->arena + off);
+        ctx->sv_warps = warps & ~7ull;
+        CK(cudaMemsetAsync(ctx->sv, 0, warps * ctx->n, ctx->stream));
+    }
     TRY(build_free_lists(ctx, r));
     uint64_t n1 = 0;
     const int k = (int)ctx->q.k;
@@ -1040,6 +1176,7 @@ namespace {
 cuts_status finish_query(cuts_ctx* ctx, const QPlan& qp, bool directed) {
     ctx->q = qp;
     ctx->q_directed = directed;
+    ctx->canon_valid = false;
     // ancestor-set reuse plan: deepest a in [2, J-1] with |bw[a]| >= 2 (an actual
     // intersection), bw[a] a subset of bw[J] and deg_Q(S[a]) <= deg_Q(S[J])
     // (undirected only)
@@ -1118,6 +1255,7 @@ cuts_status load_graph(cuts_ctx* ctx, uint32_t n, uint64_t nnz, const uint64_t* 
     uint64_t deg_bytes = align_up(rows * 4 + 4);
     if (kCtrlBytes + deg_bytes + (16u << 10) > ctx->arena_bytes) return fail(ctx, CUTS_ENOMEM, "arena too small for deg[%u]", n);
     ctx->has_graph = false;
+    ctx->canon_valid = false;
     ctx->directed = directed;
     ctx->n = n;
     ctx->nnz = nnz;
@@ -1264,20 +1402,8 @@ cuts_status cuts_level1_size(cuts_ctx* ctx, uint64_t* canonical, uint64_t* in_ra
     ctx->err.clear();
     if (!ctx->has_graph || !ctx->has_query) return fail(ctx, CUTS_ESTATE, "load_graph and set_query must precede cuts_level1_size");
     CK(cudaSetDevice(ctx->device));
-    ctx->bot = ctx->base_off;
-    ctx->top = ctx->arena_bytes & ~(kAlign - 1);
-    uint64_t off_canon, off_tmp;
-    TRY(alloc_top(ctx, (uint64_t)ctx->n * 4 + 4, &off_canon));
-    DegAtLeast pred{ctx->deg, ctx->q.qdeg[0], ctx->directed ? ctx->n : 0u, ctx->q.qdin[0]};
-    thrust::counting_iterator<uint32_t> it(0);
-    size_t tmp_bytes = 0;
-    CK(cub::DeviceSelect::If(nullptr, tmp_bytes, it, (uint32_t*)(ctx->arena + off_canon), ctx->ctrl + kNumSel,
-                             (int64_t)ctx->n, pred, ctx->stream));
-    TRY(alloc_top(ctx, tmp_bytes, &off_tmp));
-    CK(cub::DeviceSelect::If(ctx->arena + off_tmp, tmp_bytes, it, (uint32_t*)(ctx->arena + off_canon),
-                             ctx->ctrl + kNumSel, (int64_t)ctx->n, pred, ctx->stream));
-    TRY(read_ctrl(ctx));
-    const uint64_t nc = ctx->h_ctrl[kNumSel];
+    TRY(ensure_canonical(ctx));
+    const uint64_t nc = ctx->canon_n;
     const uint64_t rb = std::min(ctx->root_begin, nc), re = std::max(rb, std::min(ctx->root_end, nc));
     if (canonical) *canonical = nc;
     if (in_range) *in_range = re - rb;

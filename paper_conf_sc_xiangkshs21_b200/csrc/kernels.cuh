@@ -74,6 +74,7 @@ struct Reuse {
 
 constexpr uint64_t kTrieSrc = 1ull << 63;   // src_off flag: the source is a trie range
 constexpr uint64_t kFreeSrc = 1ull << 62;   // src_off flag: the source is a component's free list
+constexpr uint64_t kIdSrc = 1ull << 61;     // with kFreeSrc: the identity list [0, n) (degree filter in-kernel)
 constexpr uint32_t kSkip = 0xffffffffu;     // list-slot length: no list in this slot
 
 struct Graph {
@@ -104,7 +105,7 @@ enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 // ancestor range, or the set-difference searches), reported beside the model
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
             kEnumCursor = 6, kNumSel = 7, kWork = 8, kBytesOut = 9, kBytesNeed = 10, kFind = 24,
-            kDistLimbs = 56, kCtrlWords = 64 };
+            kBins = 12, kDistLimbs = 56, kCtrlWords = 64 };
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
     if (v == 0) return;
@@ -430,12 +431,13 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                                                unsigned long long* __restrict__ ctrl, int count_bytes,
                                                uint32_t batch, uint32_t qda, const uint2* __restrict__ rsrc,
                                                uint64_t* __restrict__ ord_cnt,
-                                               const uint64_t* __restrict__ ord_pos, uint32_t ord_ea) {
+                                               const uint64_t* __restrict__ ord_pos, uint32_t ord_ea,
+                                               const uint32_t* __restrict__ elist, uint32_t elist_n) {
     constexpr int VPW = 32 / G;
     constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
     constexpr int NLA = NL > 0 ? NL : 1;
     __shared__ uint32_t s_ent[2];
-    if (threadIdx.x == 0) {        // entries holding items t0 and t1-1
+    if (threadIdx.x == 0 && !elist) {        // entries holding items t0 and t1-1
         uint64_t tt[2] = {t0, t1 - 1};
         for (int z = 0; z < 2; ++z) {
             uint32_t lo = 0, hi = W - 1;
@@ -447,8 +449,9 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
         }
     }
     __syncthreads();
-    const uint32_t ea = s_ent[0];
-    const uint32_t nent = s_ent[1] - ea + 1;
+    // binned launch (CUTS_DEBUG_BINNED): the entries are an explicit list (one bin)
+    const uint32_t ea = elist ? 0u : s_ent[0];
+    const uint32_t nent = elist ? elist_n : s_ent[1] - ea + 1;
     const int lane = threadIdx.x & 31;
     const int vl = lane & (G - 1);
     const int vb = lane & ~(G - 1);
@@ -471,7 +474,7 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
             const uint32_t ei = base + bt * VPW + (uint32_t)(lane / G);
             if (!__any_sync(0xffffffffu, ei < nent)) break;
             const bool has = ei < nent;
-            const uint32_t e = ea + (has ? ei : 0);
+            const uint32_t e = elist ? __ldg(elist + (has ? ei : 0u)) : ea + (has ? ei : 0);
             // this entry's item range, clipped to [t0, t1)
             uint32_t ilo = 0, ihi = 0;
             uint64_t so = 0, obase = 0;
@@ -503,14 +506,17 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
             const bool tsrc = (so & kTrieSrc) != 0;
             // a component root's free list is already degree-filtered
             const bool fsrc = (so & kFreeSrc) != 0;
+            // ... or, when the lists did not fit the arena, the identity list [0, n): candidate = item
+            const bool isrc = fsrc && (so & kIdSrc) != 0;
+            const uint32_t qlo = isrc ? 0u : qmin;      // an identity candidate may have degree 0
             // packed CSR source (degree in the id word) only where a degree filter applies
             const bool pk = !tsrc && !fsrc && g.colx != nullptr && qd > qmin;
             const uint32_t* __restrict__ src = tsrc ? (const uint32_t*)(rsrc + (so & ~kTrieSrc))
-                                             : fsrc ? g.fre + (so & ~kFreeSrc) : (pk ? g.colx : g.col) + so;
+                                             : fsrc ? g.fre + (so & ~(kFreeSrc | kIdSrc)) : (pk ? g.colx : g.col) + so;
             const uint32_t ssh = tsrc ? 1u : 0u;
             const uint32_t umask = pk ? kPackMask : 0xffffffffu;
             // an ancestor range already passed deg >= qdeg[a]: no check needed when qdeg[J] <= qdeg[a]
-            const bool dload = qd > qmin && !pk && !fsrc && !(tsrc && qd <= qda);
+            const bool dload = qd > qlo && !pk && !(fsrc && !isrc) && !(tsrc && qd <= qda);
             const uint32_t nit = (ihi - ilo + G - 1) / G;
             unsigned long long ecnt = 0, run = 0;   // per-entry count (pass A) / ordered-write cursor
             uint32_t nit_max = nit;
@@ -579,8 +585,8 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                 for (uint32_t it = 0; it < nit_max; it += 2) {
                     const uint32_t i0 = ilo + it * G + vl, i1 = i0 + G;
                     const bool a0 = i0 < ihi, a1 = i1 < ihi;
-                    const uint32_t r0 = a0 ? __ldg(src + ((size_t)i0 << ssh)) : 0u;
-                    const uint32_t r1 = a1 ? __ldg(src + ((size_t)i1 << ssh)) : 0u;
+                    const uint32_t r0 = a0 ? (isrc ? i0 : __ldg(src + ((size_t)i0 << ssh))) : 0u;
+                    const uint32_t r1 = a1 ? (isrc ? i1 : __ldg(src + ((size_t)i1 << ssh))) : 0u;
                     const uint32_t c0 = r0 & umask, c1 = r1 & umask;
                     bool k0 = a0, k1 = a1;
 #pragma unroll
@@ -589,7 +595,7 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                         k0 = k0 && __ldg(g.deg + g.dn + c0) >= qdi;
                         k1 = k1 && __ldg(g.deg + g.dn + c1) >= qdi;
                     }
-                    if (qd > qmin) {
+                    if (qd > qlo) {
                         const uint32_t d0 = pk ? (r0 >> kPackShift) : ((k0 && dload) ? __ldg(g.deg + c0) : 0xffffffffu);
                         const uint32_t d1 = pk ? (r1 >> kPackShift) : ((k1 && dload) ? __ldg(g.deg + c1) : 0xffffffffu);
                         k0 = k0 && d0 >= qd;
@@ -678,6 +684,119 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
     }
 }
 
+// ------------------------------------------------ SV intersection (ablation)
+// Alg. 2 l.7-17, the scatter-vector intersection the paper rules
+// out for GPUs because of its O(|V| x workers) space: here every warp owns a
+// u8 scatter vector sv[|V|] in the arena (CUTS_DEBUG_SV; NEXT-2 ablation).
+// Per entry the warp (1) scatters each backward list other than the source,
+// sv[v]++ (coalesced reads, l.9-12), (2) collects: streams the source and keeps
+// c iff sv[c] == number of those lists (l.14-16) — then the degree and
+// injectivity filters and the warp-aggregated append as in k_extend — and (3)
+// clears the lists' entries again.  Levels with one list (NL = 0) have nothing
+// to intersect and use k_extend.  Count / write modes only.
+template <int J, int NL, int M>
+__global__ void __launch_bounds__(256) k_extend_sv(Graph g, QPlan q, uint64_t w0, uint32_t W,
+                                                   const uint32_t* __restrict__ path_s,
+                                                   const uint64_t* __restrict__ src_off,
+                                                   const uint64_t* __restrict__ offs,
+                                                   const uint64_t* __restrict__ lst_off,
+                                                   const uint32_t* __restrict__ lst_len,
+                                                   uint64_t t0, uint64_t t1, uint2* __restrict__ out_level,
+                                                   uint64_t cap, unsigned long long* __restrict__ ctrl,
+                                                   uint8_t* __restrict__ sv_base, uint64_t sv_stride) {
+    static_assert(NL >= 1, "SV needs a list to intersect");
+    __shared__ uint32_t s_ent[2];
+    if (threadIdx.x == 0) {
+        uint64_t tt[2] = {t0, t1 - 1};
+        for (int z = 0; z < 2; ++z) {
+            uint32_t lo = 0, hi = W - 1;
+            while (lo < hi) {
+                uint32_t mid = (lo + hi + 1) >> 1;
+                if (offs[mid] <= tt[z]) lo = mid; else hi = mid - 1;
+            }
+            s_ent[z] = lo;
+        }
+    }
+    __syncthreads();
+    const uint32_t ea = s_ent[0];
+    const uint32_t nent = s_ent[1] - ea + 1;
+    const int lane = threadIdx.x & 31;
+    const uint64_t gwarp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    uint8_t* __restrict__ sv = sv_base + gwarp * sv_stride;
+    const uint32_t qd = q.qdeg[J];
+    const uint32_t qmin = 1u;                     // undirected: list members have deg >= 1
+    unsigned long long my_count = 0;
+    unsigned int* work = (unsigned int*)(ctrl + kWork);
+    for (;;) {
+        uint32_t ei = 0;
+        if (lane == 0) ei = atomicAdd(work, 1u);
+        ei = __shfl_sync(0xffffffffu, ei, 0);
+        if (ei >= nent) break;
+        const uint32_t e = ea + ei;
+        const uint64_t o0 = offs[e], o1 = offs[e + 1];
+        const uint32_t ilo = (uint32_t)((o0 > t0 ? o0 : t0) - o0);
+        const uint32_t ihi = (uint32_t)((o1 < t1 ? o1 : t1) - o0);
+        const uint64_t so = src_off[e];
+        uint32_t path[J];
+#pragma unroll
+        for (int p = 0; p < J; ++p) path[p] = path_s[(size_t)p * W + e];
+        uint64_t lo_[NL];
+        uint32_t ln_[NL];
+        uint32_t nlists = 0;
+#pragma unroll
+        for (int x = 0; x < NL; ++x) {
+            lo_[x] = lst_off[(size_t)x * W + e];
+            ln_[x] = lst_len[(size_t)x * W + e];
+            nlists += ln_[x] != kSkip ? 1u : 0u;
+        }
+        // (1) scatter: sv[v]++ for every v of every other list (distinct within a list)
+#pragma unroll
+        for (int x = 0; x < NL; ++x) {
+            if (ln_[x] == kSkip) continue;
+            const uint32_t* l = g.col + lo_[x];
+            for (uint32_t i = lane; i < ln_[x]; i += 32) sv[__ldg(l + i)] += 1;
+            __syncwarp();
+        }
+        // (2) collect over the source items of this chunk
+        const bool pk = g.colx != nullptr && qd > qmin;
+        const uint32_t* __restrict__ src = (pk ? g.colx : g.col) + so;
+        const uint32_t umask = pk ? kPackMask : 0xffffffffu;
+        for (uint32_t b = ilo; b < ihi; b += 32) {
+            const uint32_t i = b + lane;
+            const bool act = i < ihi;
+            const uint32_t raw = act ? __ldg(src + i) : 0u;
+            const uint32_t c = raw & umask;
+            bool ok = act && sv[c] == nlists;
+#pragma unroll
+            for (int p = 0; p < J; ++p) ok = ok && path[p] != c;
+            if (qd > qmin) ok = ok && (pk ? (raw >> kPackShift) : __ldg(g.deg + c)) >= qd;
+            if (M == kCount) {
+                my_count += ok ? 1 : 0;
+            } else {
+                const unsigned m = __ballot_sync(0xffffffffu, ok);
+                unsigned long long pos0 = 0;
+                if (lane == 0 && m) pos0 = atomicAdd(ctrl + kCursor, (unsigned long long)__popc(m));
+                pos0 = __shfl_sync(0xffffffffu, pos0, 0);
+                const unsigned long long pos = pos0 + __popc(m & ((1u << lane) - 1u));
+                if (ok && pos < cap) out_level[pos] = make_uint2(c, (uint32_t)(w0 + e));
+            }
+        }
+        __syncwarp();
+        // (3) clear what (1) set
+#pragma unroll
+        for (int x = 0; x < NL; ++x) {
+            if (ln_[x] == kSkip) continue;
+            const uint32_t* l = g.col + lo_[x];
+            for (uint32_t i = lane; i < ln_[x]; i += 32) sv[__ldg(l + i)] = 0;
+        }
+        __syncwarp();
+    }
+    if (M == kCount) {
+        my_count = warp_sum(my_count);
+        if (lane == 0) add_u128(ctrl + kCountLo, my_count);
+    }
+}
+
 // ------------------------------------------------- ordered-level chunking
 // Largest eb in [ea, W] with cpos[eb] - cpos[ea] <= cap (children of entries
 // [ea, eb) fit the level chunk).  out: eb, children, items [offs[ea], offs[eb]),
@@ -695,6 +814,24 @@ __global__ void k_find_chunk(const uint64_t* __restrict__ cpos, const uint64_t* 
     out[2] = offs[ea];
     out[3] = offs[lo];
     out[4] = offs[ea + 1 <= W ? ea + 1 : W];
+}
+
+// ------------------------------------------------- binned virtual warps
+// The paper's first strategy ("group the paths based on the work
+// into bins and use virtual warps to process the bins"; kept as the NEXT-2
+// ablation CUTS_DEBUG_BINNED): entry e goes to the bin of the smallest virtual
+// warp G in {8, 16, 32} with ub(e) <= G (ub > 16: the 32-lane bin); entries
+// with no candidates are dropped.  bins[b * W + i] = i-th entry of bin b,
+// cnt[b] = bin size.
+__global__ void k_bin(const uint64_t* __restrict__ ub, uint32_t W, uint32_t* __restrict__ bins,
+                      unsigned long long* __restrict__ cnt) {
+    for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < W; e += gridDim.x * blockDim.x) {
+        const uint64_t u = ub[e];
+        if (u == 0) continue;
+        const int b = u <= 8 ? 0 : (u <= 16 ? 1 : 2);
+        const unsigned long long i = atomicAdd(cnt + b, 1ull);
+        bins[(size_t)b * W + i] = e;
+    }
 }
 
 // ---------------------------------------------------------- work donation

@@ -143,11 +143,11 @@ def test_c4_root_samples_and_chunk_invariance(cuts):
         l1, _ = ctx.level1_size()
         b0, b1 = wl.roots(l1)
         if arena is None:
-            for a, b in [r for r in _hub_ranges(g, q, (6000,)) if b0 <= r[0] < b1] + [(b0, b0 + 1), (b1 - 1, b1)]:
+            for a, b in _hub_ranges(g, q, (40000,)) + [(b0, b0 + 1), (b1 - 1, b1)]:
                 ctx.set_root_range(a, b)
                 got = ctx.count("hybrid")
                 assert got == oracle.count(g, q, root_begin=a, root_end=b), (a, b)
-        a, b = _hub_ranges(g, q, (300,))[0]
+        a, b = _hub_ranges(g, q, (2000,))[0]
         ctx.set_root_range(a, b)
         cnt = ctx.count("hybrid")
         st = ctx.stats()

@@ -44,8 +44,11 @@ def main():
     out = open(args.out, "a") if args.out else None
     flags = {f: True for f in args.debug.split(",") if f}
     for r in args.ranges:
-        a, b, den = (int(x) for x in r.split(":"))
-        rb, re = a * l1 // den, b * l1 // den
+        if r.startswith("pos:"):                 # absolute canonical positions pos:a:b
+            rb, re = (int(x) for x in r.split(":")[1:])
+        else:
+            a, b, den = (int(x) for x in r.split(":"))
+            rb, re = a * l1 // den, b * l1 // den
         for rep in range(args.reps):
             ctx.set_query(qr, qc)
             ctx.set_root_range(rb, re)

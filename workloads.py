@@ -11,12 +11,22 @@ from dataclasses import dataclass
 from inputs import rmat_graph, rmat_graph_torch, er_graph, named_query, DENSE5, SPARSE5, dense_family
 
 
+_CACHE: dict = {}
+
+
 @dataclass(frozen=True)
 class GraphSpec:
     kind: str
     params: tuple
 
     def build(self):
+        """The graph (cached per process: tests and bench reuse the same bytes)."""
+        g = _CACHE.get(self)
+        if g is None:
+            g = _CACHE[self] = self._build()
+        return g
+
+    def _build(self):
         if self.kind == "rmat":
             return rmat_graph(*self.params)
         if self.kind == "rmat_t":   # same bytes as "rmat" (tests/test_oracle.py), generated with torch
@@ -39,6 +49,7 @@ class Workload:
     parts: tuple          # ((GraphSpec, (Query, ...)), ...)
     mode: str = "hybrid"
     root_range: tuple | None = None   # (a, b, den): canonical level-1 positions [a*R/den, b*R/den)
+    min_trie_bytes: float = 0.0       # bench asserts 8 B x (deepest chunk-summed stored level) exceeds this
 
     def roots(self, l1: int):
         """Canonical root range [begin, end) for a level-1 list of size l1."""
