@@ -124,6 +124,10 @@ typedef struct {
                                   l.7-17) with a u8 sv[n] per warp in the arena,
                                   CSR lists only (no hub bitmaps, no ancestor source, no
                                   set-difference count); undirected; count/write modes      */
+#define CUTS_DEBUG_NO_PAIRS 512u /* ablation: at a count-only last level whose only list left
+                                  besides the ancestor range is the entry's own adjacency
+                                  (cliques), test every sibling pair from both ends instead
+                                  of once (the default shares each unordered pair)         */
 
 /* Create a context bound to opts->device / opts->stream / opts->arena.
  * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */

@@ -421,7 +421,8 @@ void launch_extend_g(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0
                                                                    (ctx->debug & CUTS_DEBUG_BYTES) && !w.ord_cnt ? 1 : 0, batch,
                                                                    w.ru.a ? ctx->q.qdeg[w.ru.a] : 0u,
                                                                    w.ru.lv, w.ord_cnt, w.ord_pos, w.ord_ea,
-                                                                   w.elist, w.elist_n);
+                                                                   w.elist, w.elist_n, w.ru.sym ? 2u : 1u,
+                                                                   w.ru.sym ? (uint32_t)(J - 1) : 0u);
 }
 
 template <int J, int NL, int M>
@@ -441,7 +442,8 @@ void launch_extend_nl(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t
 template <int J, int M>
 void launch_extend_t(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t0, uint64_t t1,
                      uint2* out_level, uint32_t* out_rows, uint64_t cap) {
-    const int nl = std::max(__builtin_popcount(ctx->q.bw[J]) + __builtin_popcount(ctx->q.bwi[J]) - 1, 0);   // component root: 0
+    // component root: 0; symmetric last level: one list (the entry's own)
+    const int nl = w.ru.sym ? 1 : std::max(__builtin_popcount(ctx->q.bw[J]) + __builtin_popcount(ctx->q.bwi[J]) - 1, 0);
     switch (nl) {
         case 0: launch_extend_nl<J, 0, M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
         case 1: if constexpr (J > 1) launch_extend_nl<J, (J > 1 ? 1 : 0), M>(ctx, g, w, t0, t1, out_level, out_rows, cap); break;
@@ -803,7 +805,11 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
         ctx->dfs_next[J] = w0 + w.W;
         const uint32_t a = ctx->anc[J];
         if (a && reuse_on(ctx, r) && ctx->ord[a].valid)
-            w.ru = Reuse{ctx->ord[a].lv, ctx->ord[a].cpos, ctx->ord[a].w0, ctx->ord[a].ea, a, ctx->q.bw[a]};
+            w.ru = Reuse{ctx->ord[a].lv, ctx->ord[a].cpos, ctx->ord[a].w0, ctx->ord[a].ea, a, ctx->q.bw[a],
+                         (last && !r.enumerate && a + 1 == (uint32_t)J && !ctx->directed &&
+                          (ctx->q.bw[J] & ~ctx->q.bw[a]) == (1u << a) && ctx->q.bwi[J] == 0 &&
+                          ctx->q.qdeg[J] <= ctx->q.qdeg[a] &&
+                          !(ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED))) ? 1u : 0u};
         TRY(alloc_window(ctx, J, w.W, &w));
         TRY(plan_window(ctx, r, J, w));
         if (last) {

@@ -70,6 +70,12 @@ struct Reuse {
     uint64_t ea;               // first level-a entry (window-relative) of the level a+1 chunk
     uint32_t a;                // ancestor level (0: off)
     uint32_t bwa;              // bw[a]
+    // symmetric last level ("pair sharing"): a = J-1 and the only list left
+    // to test is the entry's own N(f(S[J-1])), so sibling c_j is a child of sibling c_i iff
+    // {c_i, c_j} is an edge — the relation is symmetric.  Each entry then streams only the
+    // siblings AFTER itself and the count-only kernel doubles its sum (every unordered
+    // sibling pair tested once instead of twice)
+    uint32_t sym;
 };
 
 constexpr uint64_t kTrieSrc = 1ull << 63;   // src_off flag: the source is a trie range
@@ -288,6 +294,24 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         uint2 cur = t.lv[J][w0 + e];
         path[J - 1] = cur.x;
         uint32_t idx = cur.y;
+        if (!D && ru.sym && !count_bytes) {
+            // symmetric last level: the parent IS the ancestor (a = J-1) and the only list
+            // left is the entry's own; siblings never hold a path vertex, so no trie walk
+            const uint64_t k0 = (uint64_t)idx - ru.w0;
+            const uint64_t me = w0 + e + 1;
+            src_off[e] = me | kTrieSrc;
+            ub[e] = ru.cpos[k0 + 1] - ru.cpos[ru.ea] - me;
+            const uint32_t v = cur.x;
+            const uint32_t h = g.hub ? __ldg(g.hub + v) : kNoHub;
+            uint64_t off;
+            uint32_t len;
+            if (h != kNoHub) { off = (uint64_t)h * g.words; len = kBmFlag; }
+            else { off = g.row_ptr[v]; len = (uint32_t)(g.row_ptr[v + 1] - off); }
+            lst_off[e] = off;      // slot 0 only: the extend launch for this level has NL = 1
+            lst_len[e] = len;
+            path_s[(size_t)(J - 1) * W + e] = v;   // and reads path[J-1] only (pmin = J-1)
+            continue;
+        }
         uint32_t xa = 0;                             // index of the level-a ancestor (reuse)
 #pragma unroll
         for (int p = J - 2; p >= 0; --p) {          // trie walk
@@ -331,7 +355,13 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
 #pragma unroll
             for (int p = 0; p < J; ++p)
                 if (((bw & ~ru.bwa) >> p) & 1u) { rest_min = min(rest_min, ln_[p]); rest_sum += ln_[p]; }
-            if (trie_len <= rest_min) { trie = true; keep = bw & ~ru.bwa; }
+            if (ru.sym) {        // the siblings after this entry (w0 + e is its index in the chunk)
+                const uint64_t me = w0 + e + 1;
+                trie_len = (uint32_t)(ru.cpos[k0 + 1] - base - me);
+                trie_off = me;
+                trie = true;
+                keep = bw & ~ru.bwa;
+            } else if (trie_len <= rest_min) { trie = true; keep = bw & ~ru.bwa; }
         }
         if (need == 0) {         // component root: cross-product factor
             src_off[e] = q.foff[J] | kFreeSrc;
@@ -432,7 +462,8 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                                                uint32_t batch, uint32_t qda, const uint2* __restrict__ rsrc,
                                                uint64_t* __restrict__ ord_cnt,
                                                const uint64_t* __restrict__ ord_pos, uint32_t ord_ea,
-                                               const uint32_t* __restrict__ elist, uint32_t elist_n) {
+                                               const uint32_t* __restrict__ elist, uint32_t elist_n,
+                                               uint32_t cmul, uint32_t pmin) {
     constexpr int VPW = 32 / G;
     constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
     constexpr int NLA = NL > 0 ? NL : 1;
@@ -488,7 +519,7 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
                 so = src_off[e];
                 if (M == kWrite && ord_pos) obase = ord_pos[e] - ord_pos[ord_ea];
 #pragma unroll
-                for (int p = 0; p < J; ++p) path[p] = path_s[(size_t)p * W + e];
+                for (int p = 0; p < J; ++p) path[p] = p >= (int)pmin ? path_s[(size_t)p * W + e] : 0xffffffffu;
 #pragma unroll
                 for (int x = 0; x < NL; ++x) {
                     const uint64_t off = lst_off[(size_t)x * W + e];
@@ -671,7 +702,7 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
         }
     }
     if (M == kCount && !ord_cnt) {
-        my_count = warp_sum(my_count);
+        my_count = warp_sum(my_count) * cmul;     // cmul 2: symmetric last level (Reuse::sym)
         if (lane == 0) add_u128(ctrl + kCountLo, my_count);
     }
     if (count_bytes) {

@@ -129,11 +129,13 @@ def test_gloo_work_sharing_donations(world):
 
 
 def test_workload_root_ranges():
-    """The stated root range of C4 (first 1/16 of the canonical level-1 list) and
-    the full range of the other configs."""
-    from workloads import WORKLOADS
-    assert WORKLOADS["C4"].roots(1600) == (0, 100)
-    assert WORKLOADS["C4"].roots(17) == (0, 1)
+    """The stated root range of C4 (absolute canonical positions [13500, 14000),
+    clamped to the list) and the full range of the other configs."""
+    from workloads import WORKLOADS, Workload
+    assert WORKLOADS["C4"].roots(1834382) == (13500, 14000)
+    assert WORKLOADS["C4"].roots(13600) == (13500, 13600)
+    assert WORKLOADS["C4"].min_trie_bytes == 180e9
+    assert Workload("x", "", (), root_range=(0, 1, 16)).roots(1600) == (0, 100)
     for name in ("C1", "C2", "C3"):
         assert WORKLOADS[name].roots(1234) == (0, 1234)
     assert len(WORKLOADS["C3"].parts[0][1]) == 33

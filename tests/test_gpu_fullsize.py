@@ -157,3 +157,35 @@ def test_c4_root_samples_and_chunk_invariance(cuts):
     assert res[0][0] == res[1][0] == res[2][0]
     assert res[0][1] == res[1][1] == res[2][1]
     assert res[2][2] > res[0][2]
+
+
+def test_c4_bench_configuration_root_samples(bench_ctx):
+    """bench.py's C4 line exactly as timed (default arena, own stream, HYBRID, the
+    stated root range): the oracle on single roots sampled inside that range (the
+    lightest ones, and the range ends when light), bit-exact; and the per-root
+    counts of a short sub-range sum to the count of the sub-range."""
+    wl = WORKLOADS["C4"]
+    spec, (q,) = wl.parts[0]
+    g = spec.build()
+    bench_ctx.load_csr(g)
+    qr, qc = q.csr()
+    bench_ctx.set_query(qr, qc)
+    l1, _ = bench_ctx.level1_size()
+    b0, b1 = wl.roots(l1)
+    d = g.degrees()
+    canon = np.nonzero(d >= max(q.degrees()))[0]
+    rng = np.arange(b0, b1)
+    light = rng[np.argsort(d[canon[rng]], kind="stable")[:3]].tolist()
+    ends = [p for p in (b0, b1 - 1) if d[canon[p]] < 200]
+    for p in sorted(set(light + ends)):
+        bench_ctx.set_query(qr, qc)
+        bench_ctx.set_root_range(p, p + 1)
+        assert bench_ctx.count(wl.mode) == oracle.count(g, q, root_begin=p, root_end=p + 1), p
+    parts = 0
+    for p in range(b0, b0 + 8):
+        bench_ctx.set_query(qr, qc)
+        bench_ctx.set_root_range(p, p + 1)
+        parts += bench_ctx.count(wl.mode)
+    bench_ctx.set_query(qr, qc)
+    bench_ctx.set_root_range(b0, b0 + 8)
+    assert bench_ctx.count(wl.mode) == parts

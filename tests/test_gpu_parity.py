@@ -113,7 +113,7 @@ def test_ancestor_reuse_chunked(cuts, arena_kib):
     for q in qs:
         want, lv = oracle.count(g, q, levels=True)
         _set(c, q)
-        for flags in (0, 4):
+        for flags in (0, 4, 512):        # default (pair-shared last level), no reuse, no pair sharing
             c.lib.cuts_set_debug(c.h, flags)
             assert c.count("hybrid") == want, (arena_kib, q.name, flags)
             assert c.stats()["level_size"] == lv, (arena_kib, q.name, flags)
@@ -534,7 +534,8 @@ def test_next2_binned_and_sv_variants(cuts, flag):
             want, lv = oracle.count(g, q, levels=True)
             _set(c, q)
             c.set_debug(**{flag: True})
-            for mode in ("hybrid", "bfs") if arena > (1 << 20) else ("hybrid",):
+            bfs_fits = arena > (1 << 20) and 8 * max(lv) < arena // 8
+            for mode in ("hybrid", "bfs") if bfs_fits else ("hybrid",):
                 assert c.count(mode) == want, (flag, arena, q.name, mode)
                 assert c.stats()["level_size"] == lv, (flag, arena, q.name, mode)
             if flag == "binned" and want <= 1_000_000 and arena > (1 << 20):

@@ -11,8 +11,13 @@ k_extend milliseconds.  Variants (all give the same counts; checked here):
   sv_hubs   : + SV-style bitmaps for hub lists (Alg. 2 l.7-17)
   packed    : + packed (id | degree) stream (degree filter without a gather)
   reuse     : + ancestor-set source
-  full      : + set-difference count at a single-list degree-free last level
-              (the product default)
+  fastcount : + set-difference count at a single-list degree-free last level
+  full      : + pair-shared symmetric last level (the product default)
+Side variants (NEXT-2, compare with the chain member named):
+  binned    : fastcount with binned virtual warps at the last level
+              instead of the single bin
+  sv        : the per-warp scatter-vector intersection (Alg. 2 l.7-17) on CSR
+              lists (compare with packed: same source, no bitmaps/reuse)
 """
 import argparse
 import json
@@ -33,8 +38,11 @@ VARIANTS = [  # (name, hub threshold, debug kwargs)
     ("short_c", None, dict(no_pack=True, no_reuse=True, no_fast_count=True)),
     ("sv_hubs", 0, dict(no_pack=True, no_reuse=True, no_fast_count=True)),
     ("packed", 0, dict(no_reuse=True, no_fast_count=True)),
-    ("reuse", 0, dict(no_fast_count=True)),
+    ("reuse", 0, dict(no_fast_count=True, no_pairs=True)),
+    ("fastcount", 0, dict(no_pairs=True)),
     ("full", 0, dict()),
+    ("binned", 0, dict(no_pairs=True, binned=True)),
+    ("sv", None, dict(sv=True)),
 ]
 
 
@@ -67,6 +75,9 @@ def main():
                 ctx.set_debug(timing=True, **dbg)
                 best, st, c = None, None, None
                 for _ in range(args.reps):
+                    ctx.set_query(qr, qc)
+                    if wl.root_range is not None:
+                        ctx.set_root_range(*wl.roots(ctx.level1_size()[0]))
                     torch.cuda.synchronize()
                     t = time.time()
                     c = ctx.count(wl.mode)

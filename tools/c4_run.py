@@ -41,8 +41,7 @@ def main():
     qr, qc = q.csr()
     ctx.set_query(qr, qc)
     l1, _ = ctx.level1_size()
-    rr = C4.root_range if not args.den else (0, 1, args.den)
-    b, e = rr[0] * l1 // rr[2], rr[1] * l1 // rr[2]
+    b, e = C4.roots(l1) if not args.den else (0, l1 // args.den)
     rec = {"graph": spec.name, "n": g.n, "m": g.m, "gen_s": round(gen_s, 1), "query": q.name,
            "level1_canonical": l1, "root_range": [b, e], "arena_bytes": ctx.arena.numel()}
     if not args.skip_bfs:

@@ -26,7 +26,7 @@ for st in "$@"; do
              --log-file gpurun_out/${tag}_launches.csv python bench.py --steps 1 --warmup 0 --no-cpu-baseline $arg \
              > gpurun_out/${tag}_ncu_launch.log 2>&1; tail -3 gpurun_out/${tag}_ncu_launch.log ;;
     ncu_full) IFS=: read -r rx skip rest <<< "$arg"
-             timeout -k 10 1800 ncu --set full --clock-control none --import-source on -k "regex:${rx}" -s ${skip:-0} -c 1 \
+             timeout -k 10 1800 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k "regex:${rx}" -s ${skip:-0} -c 1 \
              -o gpurun_out/${tag}_full -f $rest > gpurun_out/${tag}_ncu_full.log 2>&1; tail -5 gpurun_out/${tag}_ncu_full.log ;;
     *) echo "unknown step $name" ;;
   esac

@@ -52,10 +52,13 @@ class Workload:
     min_trie_bytes: float = 0.0       # bench asserts 8 B x (deepest chunk-summed stored level) exceeds this
 
     def roots(self, l1: int):
-        """Canonical root range [begin, end) for a level-1 list of size l1."""
+        """Canonical root range [begin, end) for a level-1 list of size l1
+        (den == 0: a and b are absolute positions)."""
         if self.root_range is None:
             return 0, l1
         a, b, den = self.root_range
+        if den == 0:
+            return min(a, l1), min(b, l1)
         return a * l1 // den, b * l1 // den
 
 
@@ -87,15 +90,20 @@ C3 = Workload(
     ((C3_GRAPH, tuple(dense_family(6) + dense_family(7) + dense_family(8))),))
 
 # configs[3]: 8-vertex dense query on R-MAT scale 22 forcing hybrid BFS/DFS chunking
-# beyond 180 GB.  R-MAT(22, 16, .50, .20, .20), K8, restricted to the first 1/16 of
-# the canonical level-1 list (stated, as SURVEY §8.d allows).  Measured
-# (profiles/r01_c4_run_reuse.json): levels 1.1e5 / 7.8e6 / 3.3e7 / 4.0e8 / 7.6e9 /
-# 1.6e11 / 3.5e12, count 7.33e13 — the deepest stored level alone would be 28 TB of
-# 8 B trie entries (BFS stops with CUTS_ENOMEM at level 5), HYBRID finishes in
-# 1,604 s on one B200.
+# beyond 180 GB: K8 on R-MAT(22, 16, .50, .20, .20) (n 4,194,304, 66.9 M edges, CSR
+# 547 MB), restricted to the stated canonical level-1 positions [13500, 14000) of
+# 1,834,382 (SURVEY §8.d allows a stated root range).  Calibrated in round 2
+# (profiles/r02b_c4sweep.jsonl): work is concentrated on the hub roots (tiers of
+# degree ~45 K, ~21 K, ~9.4 K, ~4 K); this range holds one ~9.4 K-degree hub
+# (position 13997) plus 499 ordinary roots: levels 9.1e3 / 4.0e5 / 8.3e6 / 1.7e8 /
+# 3.1e9 / 5.2e10 (the deepest stored level alone = 415 GB of 8 B trie entries, so
+# BFS cannot hold it and HYBRID chunking is on the timed path) and 8.0e11
+# embeddings per step.  The round-1 range [0, 1/16) holds two ~21 K hubs and took
+# 1,604 s per pass — too long for a 25-step driver run.
 C4_GRAPH = GraphSpec("rmat_t", (22, 16, 0.50, 0.20, 0.20, 1))
 C4 = Workload(
-    "C4", "K8 on R-MAT(22,16,.50,.20,.20), canonical roots [0, 1/16); hybrid count beyond 180 GB",
-    ((C4_GRAPH, (dense_family(8)[0],)),), root_range=(0, 1, 16))
+    "C4", "K8 on R-MAT(22,16,.50,.20,.20), canonical roots [13500, 14000) (one ~9.4K-degree hub); "
+          "hybrid count, deepest stored level > 180 GB",
+    ((C4_GRAPH, (dense_family(8)[0],)),), root_range=(13500, 14000, 0), min_trie_bytes=180e9)
 
 WORKLOADS = {"C1": C1, "C2": C2, "C3": C3, "C4": C4}
