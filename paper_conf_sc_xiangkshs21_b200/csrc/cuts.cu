@@ -99,7 +99,7 @@ struct cuts_ctx {
     // written ordered (children contiguous per parent, exact offsets kept)
     uint32_t anc[kMaxK + 1] = {};
     uint32_t need_ord = 0;
-    struct OrdState { const uint64_t* cpos; uint64_t w0; uint64_t ea; const uint2* lv; bool valid; };
+    struct OrdState { const uint64_t* cpos; uint64_t w0; uint64_t ea; const uint2* lv; bool valid; uint64_t eb; };
     OrdState ord[kMaxK + 1] = {};
     // CUTS_DEBUG_SV: per-warp u8 scatter vectors of n entries (zeroed; kernels leave them clean)
     uint8_t* sv = nullptr;
@@ -769,7 +769,7 @@ cuts_status hybrid_ordered(cuts_ctx* ctx, Run& r, int J, Window& w) {
                 wb.ord_ea = ea;
                 TRY(extend_range(ctx, r, J, wb, i0, i1, kWrite, out, size));
                 ctx->st.level_size[J + 1] += size;
-                ctx->ord[J] = {w.cpos, w.w0, ea, out, true};
+                ctx->ord[J] = {w.cpos, w.w0, ea, out, true, eb};
                 r.t.lv[J + 1] = out;
                 TRY(hybrid_level(ctx, r, J + 1, size));
                 ctx->ord[J].valid = false;
@@ -787,10 +787,51 @@ cuts_status hybrid_ordered(cuts_ctx* ctx, Run& r, int J, Window& w) {
     return CUTS_OK;
 }
 
+// symmetric last level (Reuse::sym conditions): is level J's count a pair count over
+// sibling groups of the ordered level-(J-1) chunk?
+bool sym_last(const cuts_ctx* ctx, const Run& r, int J) {
+    const uint32_t a = ctx->anc[J];
+    return J == (int)ctx->q.k - 1 && a && a + 1 == (uint32_t)J && reuse_on(ctx, r) && ctx->ord[a].valid &&
+           !r.enumerate && !ctx->directed && (ctx->q.bw[J] & ~ctx->q.bw[a]) == (1u << a) && ctx->q.bwi[J] == 0 &&
+           ctx->q.qdeg[J] <= ctx->q.qdeg[a] && !(ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED));
+}
+
+// the whole level-J chunk in one k_pairs launch (no plan windows); CUTS_DEBUG_BYTES
+// runs take the windowed path instead, whose k_plan counts the §8.d model per entry
+cuts_status pairs_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
+    const auto& o = ctx->ord[J - 1];
+    const double m = (double)N / (double)std::max<uint64_t>(o.eb - o.ea, 1);   // siblings per group
+    const double avg = m / 2;                                                  // tested per entry
+    int e0 = -1;
+    CK(cudaMemsetAsync(ctx->ctrl + kWork, 0, sizeof(unsigned long long), ctx->stream));
+    if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
+    auto go = [&](auto kern, int G) {
+        static int occ[3] = {0, 0, 0};
+        int& oc = occ[G == 8 ? 0 : (G == 16 ? 1 : 2)];
+        if (!oc) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&oc, kern, 256, 0); if (oc < 1) oc = 1; }
+        const uint64_t grid = std::min<uint64_t>((uint64_t)ctx->num_sms * oc, (N * G + 255) / 256 + 1);
+        const uint32_t batch = (uint32_t)std::min(256.0, std::max(2.0, 2048.0 / std::max(avg, 1.0) / (32 / G)));
+        kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, ctx->ctrl, batch);
+    };
+    if (avg >= 48) go(k_pairs<32>, 32);
+    else if (avg >= 12) go(k_pairs<16>, 16);
+    else go(k_pairs<8>, 8);
+    CK(cudaGetLastError());
+    if (ctx->debug & CUTS_DEBUG_TIMING) {
+        const int e1 = next_event(ctx);
+        CK(cudaEventRecord(ctx->ev_pool[e1], ctx->stream));
+        ctx->ev_ext.push_back({e0, e1});
+    }
+    ctx->st.chunks++;
+    ctx->st.launches += 2;
+    return CUTS_OK;
+}
+
 cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     const int k = (int)ctx->q.k;
     const bool last = (J == k - 1);
     const uint64_t top_save = ctx->top;
+    if (last && !(ctx->debug & CUTS_DEBUG_BYTES) && sym_last(ctx, r, J)) return pairs_level(ctx, r, J, N);
     const bool ordered = !last && reuse_on(ctx, r) && ((ctx->need_ord >> J) & 1u);
     ctx->dfs_on[J] = true;
     ctx->dfs_next[J] = 0;
@@ -806,10 +847,7 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
         const uint32_t a = ctx->anc[J];
         if (a && reuse_on(ctx, r) && ctx->ord[a].valid)
             w.ru = Reuse{ctx->ord[a].lv, ctx->ord[a].cpos, ctx->ord[a].w0, ctx->ord[a].ea, a, ctx->q.bw[a],
-                         (last && !r.enumerate && a + 1 == (uint32_t)J && !ctx->directed &&
-                          (ctx->q.bw[J] & ~ctx->q.bw[a]) == (1u << a) && ctx->q.bwi[J] == 0 &&
-                          ctx->q.qdeg[J] <= ctx->q.qdeg[a] &&
-                          !(ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED))) ? 1u : 0u};
+                         sym_last(ctx, r, J) ? 1u : 0u};
         TRY(alloc_window(ctx, J, w.W, &w));
         TRY(plan_window(ctx, r, J, w));
         if (last) {

@@ -715,6 +715,99 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
     }
 }
 
+// ------------------------------------------- symmetric last level: pair count
+// The count-only last level J = k-1 when the level J-1 -> J extension was written
+// ordered and the only condition left is adjacency to the entry itself (cliques;
+// Reuse::sym): entry e (vertex c_e, parent p) of the level-J chunk has as
+// candidates its siblings, the children of p, stored contiguously and ascending;
+// sibling c_j is a child of e iff {c_e, c_j} is an edge (the degree filter and
+// injectivity are implied: DESIGN.md §7).  Each unordered sibling pair is tested
+// once — e tests only the siblings after itself — and the sum is doubled.  No
+// plan pass: virtual warps of G lanes take entries straight from the chunk, read
+// the sibling range end from the parent's scan slot and test membership in N(c_e)
+// by the hub bitmap or a cursor-narrowed binary search (candidates ascend).
+//   lv     : the level-J chunk (.x = vertex, .y = index of the parent in level J-1)
+//   cpos   : level J-1 window's exclusive scan of child counts; cw0 = that window's
+//            start (parent index p -> slot p - cw0); cea = slot of the chunk's first parent
+template <int G>
+__global__ void __launch_bounds__(256, 6) k_pairs(Graph g, const uint2* __restrict__ lv, uint64_t nent,
+                                                  const uint64_t* __restrict__ cpos, uint64_t cw0, uint64_t cea,
+                                                  unsigned long long* __restrict__ ctrl, uint32_t batch) {
+    const uint64_t cbase = cpos[cea];
+    constexpr int VPW = 32 / G;
+    constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
+    const int lane = threadIdx.x & 31;
+    const int vl = lane & (G - 1);
+    const int vb = lane & ~(G - 1);
+    unsigned long long my_count = 0;
+    unsigned long long* work = ctrl + kWork;
+    for (;;) {
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(work, (unsigned long long)VPW * batch);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (base >= nent) break;
+#pragma unroll 1
+        for (uint32_t bt = 0; bt < batch; ++bt) {
+            const uint64_t e = base + (uint64_t)bt * VPW + (uint64_t)(lane / G);
+            if (!__any_sync(0xffffffffu, e < nent)) break;
+            const bool has = e < nent;
+            uint32_t v = 0, len = 0;
+            uint64_t end = 0;
+            const uint32_t* lb = g.col;
+            bool bmp = false;
+            if (has) {
+                const uint2 x = lv[e];
+                v = x.x;
+                end = cpos[x.y - cw0 + 1] - cbase;
+                const uint32_t h = g.hub ? __ldg(g.hub + v) : kNoHub;
+                if (h != kNoHub) {
+                    bmp = true;
+                    lb = g.bm + (uint64_t)h * g.words;
+                } else {
+                    const uint64_t b = g.row_ptr[v];
+                    lb = g.col + b;
+                    len = (uint32_t)(g.row_ptr[v + 1] - b);
+                }
+            }
+            const uint32_t nit = has ? (uint32_t)((end - (e + 1) + G - 1) / G) : 0u;
+            uint32_t nit_max = nit;
+            if (VPW > 1) {
+#pragma unroll
+                for (int o = 16; o >= G; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
+            }
+            for (uint32_t it = 0; it < nit_max; ++it) {
+                const uint64_t j = e + 1 + (uint64_t)it * G + vl;
+                const bool act = has && j < end;
+                const uint32_t c = act ? lv[j].x : 0u;
+                bool ok = act;
+                if (bmp && act) ok = (__ldg(lb + (c >> 5)) >> (c & 31)) & 1u;   // hub: one bitmap probe
+                const bool pend = act && !bmp;
+                const unsigned pw = __ballot_sync(0xffffffffu, pend);
+                uint32_t pos = 0;
+                if (pend) {          // branch-free lower bound from the cursor
+                    const uint32_t* b0 = lb;
+                    uint32_t l = len;
+                    while (l > 1) {
+                        const uint32_t half = l >> 1;
+                        b0 = (__ldg(b0 + half - 1) < c) ? b0 + half : b0;
+                        l -= half;
+                    }
+                    ok = len > 0 && __ldg(b0) == c;
+                    pos = (uint32_t)(b0 - lb);
+                }
+                // siblings ascend with the lane: the highest pending lane bounds the cursor
+                const unsigned pv = (pw >> vb) & kGMask;
+                const int hl = pv ? vb + 31 - __clz(pv) : lane;
+                const uint32_t mpos = __shfl_sync(0xffffffffu, pos, hl);
+                if (pv) { lb += mpos; len -= mpos; }
+                my_count += ok ? 1 : 0;
+            }
+        }
+    }
+    my_count = warp_sum(my_count) * 2ull;          // every unordered pair counted once
+    if (lane == 0) add_u128(ctrl + kCountLo, my_count);
+}
+
 // ------------------------------------------------ SV intersection (ablation)
 // Alg. 2 l.7-17, the scatter-vector intersection the paper rules
 // out for GPUs because of its O(|V| x workers) space: here every warp owns a
