@@ -189,7 +189,7 @@ def run_ours(args):
 
     def step(timing=False):
         """One pass over every (graph, query): (local count, launches, ms_extend, extend launches, level sizes)."""
-        total, launches, ms_ext, n_ext = 0, 0, 0.0, 0
+        total, launches, ms_ext, n_ext, fused = 0, 0, 0.0, 0, 0
         levels = [0] * 9
         ctx.set_debug(timing=timing)
         pass_id[0] += 1
@@ -203,9 +203,10 @@ def run_ours(args):
                     launches += st["launches"]
                     ms_ext += st["ms_extend"]
                     n_ext += st["extend_launches"]
+                    fused |= st["fused_levels"]
                     for j, v in enumerate(st["level_size"]):
                         levels[j] += v
-        return total, launches, ms_ext, n_ext, levels
+        return total, launches, ms_ext, n_ext, (levels, fused)
 
     def barrier():
         torch.cuda.synchronize(dev)
@@ -218,7 +219,7 @@ def run_ours(args):
     barrier()
     sampler = ClockSampler(local)
     sampler.start()
-    times, counts, launches, ms_ext, n_ext, levels = [], [], 0, 0.0, 0, None
+    times, counts, launches, ms_ext, n_ext, levels = [], [], 0, 0.0, 0, ([], 0)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for _ in range(args.steps):
         flush.fill_(1)                      # evict L2 between timed steps
@@ -238,10 +239,13 @@ def run_ours(args):
     local_count = counts[-1]
     step_ms = D.allreduce_max(step_ms_local, device=dev)            # max over ranks
     step_count = D.allreduce_count(local_count, device=dev, ctx=ctx)   # the library's NCCL sum (N > 1)
+    levels, fused = levels
     levels = [D.allreduce_count(v, device=dev) for v in levels]      # chunk- and rank-summed level sizes
     value = step_count / (step_ms / 1e3)
     nq = sum(len(qs) for _, qs in graphs)
-    deepest = max(levels[1:max(q.k for _, qs in graphs for q in qs)]) if levels else 0
+    kmax = max(q.k for _, qs in graphs for q in qs)
+    stored = [j for j in range(1, kmax) if not (fused >> j) & 1]     # levels written to the trie arena
+    deepest = max((levels[j] for j in stored), default=0)
     if wl.min_trie_bytes and 8 * deepest <= wl.min_trie_bytes:
         raise SystemExit(f"workload {wl.name}: deepest stored level {deepest} entries = {8 * deepest:.3e} B "
                          f"<= {wl.min_trie_bytes:.3e} B — the root range no longer forces HYBRID chunking")
@@ -309,8 +313,9 @@ def run_ours(args):
                    "graphs": [s.name for s, _ in wl.parts], "embeddings_per_step": step_count,
                    "mode": wl.mode, "l2": "flushed between timed steps (256 MiB write)",
                    "root_range": (list(wl.root_range) if wl.root_range else None),
-                   "level_size_per_step": levels, "deepest_stored_level": deepest,
-                   "bfs_trie_bytes_at_deepest_level": 8 * deepest,
+                   "level_size_per_step": levels, "stored_levels": stored,
+                   "deepest_stored_level_entries": deepest, "deepest_stored_level_bytes": 8 * deepest,
+                   "bfs_trie_bytes_at_largest_level": 8 * max(levels[1:kmax], default=0),
                    "parallelism": (f"NCCL world {world} via cuts_set_dist; dynamic root-chunk queue "
                                    f"({args.chunks_per_rank} chunks/rank/query)"
                                    + (" + Alg. 3 prefix donations (store control plane, gloo host data plane)"

@@ -99,6 +99,9 @@ typedef struct {
     uint64_t free_identity;            /* disconnected Q: 1 if the component roots streamed the
                                           identity list [0, n) with an in-kernel degree
                                           filter (the filtered lists did not fit the arena)  */
+    uint64_t fused_levels;             /* bit j: level j was (at least partly) never stored —
+                                          the local-rows tail counts it from the level j-1
+                                          sibling rows (level_size[j] stays exact)           */
 } cuts_stats;
 
 /* debug / instrumentation flags for cuts_set_debug */
@@ -128,6 +131,10 @@ typedef struct {
                                   besides the ancestor range is the entry's own adjacency
                                   (cliques), test every sibling pair from both ends instead
                                   of once (the default shares each unordered pair)         */
+#define CUTS_DEBUG_NO_LR 1024u /* ablation: no local rows — the last two levels of a
+                                  clique-like tail go through the trie pipeline (ordered
+                                  write of level k-1, pair count) instead of 64-bit sibling
+                                  adjacency rows of the level-(k-2) groups                  */
 
 /* Create a context bound to opts->device / opts->stream / opts->arena.
  * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */

@@ -796,6 +796,62 @@ bool sym_last(const cuts_ctx* ctx, const Run& r, int J) {
            ctx->q.qdeg[J] <= ctx->q.qdeg[a] && !(ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED));
 }
 
+// local rows: level J = k-2 of a clique-like tail — the ordered level-J
+// chunk's sibling groups carry both remaining extensions (J -> J+1 and the count)
+bool lr_level(const cuts_ctx* ctx, const Run& r, int J) {
+    const int k = (int)ctx->q.k;
+    if (J != k - 2 || J < 3 || r.enumerate || ctx->directed || !reuse_on(ctx, r)) return false;
+    if (ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED | CUTS_DEBUG_BYTES | CUTS_DEBUG_NO_LR)) return false;
+    auto sym = [&](int L) {
+        const uint32_t a = ctx->anc[L];
+        return a && a + 1 == (uint32_t)L && (ctx->q.bw[L] & ~ctx->q.bw[a]) == (1u << a) && ctx->q.bwi[L] == 0 &&
+               ctx->q.qdeg[L] <= ctx->q.qdeg[a];
+    };
+    return sym(J) && sym(J + 1) && ctx->ord[J - 1].valid;
+}
+
+// rows + bit algebra over the whole level-J chunk; returns the number of entries in
+// groups too large for 64-bit rows (the windowed pipeline then takes those)
+cuts_status lr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large) {
+    const auto& o = ctx->ord[J - 1];
+    uint64_t off;
+    TRY(alloc_top(ctx, N * 8, &off));
+    unsigned long long* R = (unsigned long long*)(ctx->arena + off);
+    CK(cudaMemsetAsync(R, 0, N * 8, ctx->stream));
+    CK(cudaMemsetAsync(ctx->ctrl + kWork, 0, sizeof(unsigned long long), ctx->stream));
+    CK(cudaMemsetAsync(ctx->ctrl + kLrLarge, 0, sizeof(unsigned long long), ctx->stream));
+    const double m = (double)N / (double)std::max<uint64_t>(o.eb - o.ea, 1);
+    const double avg = m / 2;
+    int e0 = -1;
+    if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
+    auto go = [&](auto kern, int G) {
+        static int occ[3] = {0, 0, 0};
+        int& oc = occ[G == 8 ? 0 : (G == 16 ? 1 : 2)];
+        if (!oc) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&oc, kern, 256, 0); if (oc < 1) oc = 1; }
+        const uint64_t grid = std::min<uint64_t>((uint64_t)ctx->num_sms * oc, (N * G + 255) / 256 + 1);
+        const uint32_t batch = (uint32_t)std::min(256.0, std::max(2.0, 2048.0 / std::max(avg, 1.0) / (32 / G)));
+        kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl, batch);
+    };
+    if (avg >= 48) go(k_lr_rows<32>, 32);
+    else if (avg >= 12) go(k_lr_rows<16>, 16);
+    else go(k_lr_rows<8>, 8);
+    CK(cudaGetLastError());
+    const unsigned grid = (unsigned)std::min<uint64_t>((N + 255) / 256, (uint64_t)ctx->num_sms * 16);
+    k_lr_count<<<grid, 256, 0, ctx->stream>>>(r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl);
+    CK(cudaGetLastError());
+    if (ctx->debug & CUTS_DEBUG_TIMING) {
+        const int e1 = next_event(ctx);
+        CK(cudaEventRecord(ctx->ev_pool[e1], ctx->stream));
+        ctx->ev_ext.push_back({e0, e1});
+    }
+    CK(cudaMemcpyAsync(ctx->h_ctrl + kLrLarge, ctx->ctrl + kLrLarge, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    *large = ctx->h_ctrl[kLrLarge];
+    ctx->st.chunks++;
+    ctx->st.launches += 2;
+    return CUTS_OK;
+}
+
 // the whole level-J chunk in one k_pairs launch (no plan windows); CUTS_DEBUG_BYTES
 // runs take the windowed path instead, whose k_plan counts the §8.d model per entry
 cuts_status pairs_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
@@ -832,6 +888,15 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     const bool last = (J == k - 1);
     const uint64_t top_save = ctx->top;
     if (last && !(ctx->debug & CUTS_DEBUG_BYTES) && sym_last(ctx, r, J)) return pairs_level(ctx, r, J, N);
+    bool skip_small = false;
+    if (lr_level(ctx, r, J) && free_bytes(ctx) >= N * 8 + (1u << 20)) {   // rows: 8 B per entry
+        uint64_t large = 0;
+        TRY(lr_chunk(ctx, r, J, N, &large));
+        ctx->top = top_save;
+        ctx->st.fused_levels |= 1ull << (J + 1);   // level k-1 of the small groups is never stored
+        if (large == 0) return CUTS_OK;       // every group was small: nothing left at this level
+        skip_small = true;
+    }
     const bool ordered = !last && reuse_on(ctx, r) && ((ctx->need_ord >> J) & 1u);
     ctx->dfs_on[J] = true;
     ctx->dfs_next[J] = 0;
@@ -847,7 +912,7 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
         const uint32_t a = ctx->anc[J];
         if (a && reuse_on(ctx, r) && ctx->ord[a].valid)
             w.ru = Reuse{ctx->ord[a].lv, ctx->ord[a].cpos, ctx->ord[a].w0, ctx->ord[a].ea, a, ctx->q.bw[a],
-                         sym_last(ctx, r, J) ? 1u : 0u};
+                         sym_last(ctx, r, J) ? 1u : 0u, skip_small ? 1u : 0u};
         TRY(alloc_window(ctx, J, w.W, &w));
         TRY(plan_window(ctx, r, J, w));
         if (last) {
@@ -1187,6 +1252,7 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
         ctx->st.count_hi = ctx->h_ctrl[kCountHi];
     }
     if (k > 1) ctx->st.level_size[k] = ctx->st.count_lo;
+    if (k >= 5) ctx->st.level_size[k - 1] += ctx->h_ctrl[kLrLevel];   // local rows: |L_{k-1}| of the small groups
     ctx->st.alg_bytes_plan = ctx->h_ctrl[kBytesPlan];
     ctx->st.alg_bytes_extend = ctx->h_ctrl[kBytesExt] + ctx->h_ctrl[kBytesOut];
     ctx->st.alg_bytes_extend_needed = ctx->h_ctrl[kBytesNeed] + ctx->h_ctrl[kBytesOut];

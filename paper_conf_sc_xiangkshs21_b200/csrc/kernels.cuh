@@ -76,6 +76,9 @@ struct Reuse {
     // siblings AFTER itself and the count-only kernel doubles its sum (every unordered
     // sibling pair tested once instead of twice)
     uint32_t sym;
+    // local rows took this level's small sibling groups (<= 64 members): k_plan gives
+    // their entries no candidates (ub = 0) so the windowed pipeline only sees the rest
+    uint32_t skip_small;
 };
 
 constexpr uint64_t kTrieSrc = 1ull << 63;   // src_off flag: the source is a trie range
@@ -111,7 +114,7 @@ enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 // ancestor range, or the set-difference searches), reported beside the model
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
             kEnumCursor = 6, kNumSel = 7, kWork = 8, kBytesOut = 9, kBytesNeed = 10, kFind = 24,
-            kBins = 12, kDistLimbs = 56, kCtrlWords = 64 };
+            kBins = 12, kLrLevel = 15, kLrLarge = 29, kDistLimbs = 56, kCtrlWords = 64 };
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
     if (v == 0) return;
@@ -311,6 +314,14 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
             lst_len[e] = len;
             path_s[(size_t)(J - 1) * W + e] = v;   // and reads path[J-1] only (pmin = J-1)
             continue;
+        }
+        if (ru.skip_small) {
+            const uint64_t k0 = (uint64_t)idx - ru.w0;   // the parent is the ancestor (a = J-1)
+            if (ru.cpos[k0 + 1] - ru.cpos[k0] <= 64) {
+                ub[e] = 0;
+                src_off[e] = 0;
+                continue;
+            }
         }
         uint32_t xa = 0;                             // index of the level-a ancestor (reuse)
 #pragma unroll
@@ -806,6 +817,133 @@ __global__ void __launch_bounds__(256, 6) k_pairs(Graph g, const uint2* __restri
     }
     my_count = warp_sum(my_count) * 2ull;          // every unordered pair counted once
     if (lane == 0) add_u128(ctrl + kCountLo, my_count);
+}
+
+// ------------------------------------------------ local rows (clique tail)
+// The last two extension levels of a clique-like tail ("local rows"):
+// level-b entries (b = k-2) come in sibling groups S_q (the ordered children of a
+// level-(b-1) entry q, contiguous, ascending).  When both remaining extensions only
+// add adjacency to the newest vertex (Reuse::sym conditions at b and at b+1), then
+//   children(e_i)        = S_q[R_i]            with R_i = {j : S_q[j] in N(S_q[i])}
+//   children((e_i, c_j)) = S_q[R_i & R_j]
+// so for a group with m <= 64 members the 64-bit rows R_i are all the intersection
+// work: |L_{b+1}| += popc(R_i) and the count += sum_{j in R_i} popc(R_i & R_j).
+// k_lr_rows tests every unordered sibling pair once (hub bitmap or cursor-narrowed
+// binary search, as k_pairs) and sets both bits; k_lr_count does the bit algebra.
+// Groups with m > 64 are left to the ordinary pipeline (Reuse::skip_small).
+template <int G>
+__global__ void __launch_bounds__(256, 6) k_lr_rows(Graph g, const uint2* __restrict__ lv, uint64_t nent,
+                                                    const uint64_t* __restrict__ cpos, uint64_t cw0, uint64_t cea,
+                                                    unsigned long long* __restrict__ R,
+                                                    unsigned long long* __restrict__ ctrl, uint32_t batch) {
+    constexpr int VPW = 32 / G;
+    constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
+    const uint64_t cbase = cpos[cea];
+    const int lane = threadIdx.x & 31;
+    const int vl = lane & (G - 1);
+    const int vb = lane & ~(G - 1);
+    unsigned long long large = 0;
+    unsigned long long* work = ctrl + kWork;
+    for (;;) {
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(work, (unsigned long long)VPW * batch);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (base >= nent) break;
+#pragma unroll 1
+        for (uint32_t bt = 0; bt < batch; ++bt) {
+            const uint64_t e = base + (uint64_t)bt * VPW + (uint64_t)(lane / G);
+            if (!__any_sync(0xffffffffu, e < nent)) break;
+            bool has = e < nent;
+            uint32_t v = 0, len = 0;
+            uint64_t g0 = 0, end = 0;
+            const uint32_t* lb = g.col;
+            bool bmp = false;
+            if (has) {
+                const uint2 x = lv[e];
+                v = x.x;
+                g0 = cpos[x.y - cw0] - cbase;
+                end = cpos[x.y - cw0 + 1] - cbase;
+                if (end - g0 > 64) {             // large group: the ordinary pipeline takes it
+                    if (vl == 0) large += 1;
+                    has = false;
+                } else {
+                    const uint32_t h = g.hub ? __ldg(g.hub + v) : kNoHub;
+                    if (h != kNoHub) {
+                        bmp = true;
+                        lb = g.bm + (uint64_t)h * g.words;
+                    } else {
+                        const uint64_t b = g.row_ptr[v];
+                        lb = g.col + b;
+                        len = (uint32_t)(g.row_ptr[v + 1] - b);
+                    }
+                }
+            }
+            const uint32_t nit = has ? (uint32_t)((end - (e + 1) + G - 1) / G) : 0u;
+            uint32_t nit_max = nit;
+            if (VPW > 1) {
+#pragma unroll
+                for (int o = 16; o >= G; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
+            }
+            unsigned long long row = 0;
+            for (uint32_t it = 0; it < nit_max; ++it) {
+                const uint64_t j = e + 1 + (uint64_t)it * G + vl;
+                const bool act = has && j < end;
+                const uint32_t c = act ? lv[j].x : 0u;
+                bool ok = act;
+                if (bmp && act) ok = (__ldg(lb + (c >> 5)) >> (c & 31)) & 1u;
+                const bool pend = act && !bmp;
+                const unsigned pw = __ballot_sync(0xffffffffu, pend);
+                uint32_t pos = 0;
+                if (pend) {
+                    const uint32_t* b0 = lb;
+                    uint32_t l = len;
+                    while (l > 1) {
+                        const uint32_t half = l >> 1;
+                        b0 = (__ldg(b0 + half - 1) < c) ? b0 + half : b0;
+                        l -= half;
+                    }
+                    ok = len > 0 && __ldg(b0) == c;
+                    pos = (uint32_t)(b0 - lb);
+                }
+                const unsigned pv = (pw >> vb) & kGMask;
+                const int hl = pv ? vb + 31 - __clz(pv) : lane;
+                const uint32_t mpos = __shfl_sync(0xffffffffu, pos, hl);
+                if (pv) { lb += mpos; len -= mpos; }
+                if (ok) {                          // the pair {i, j}: bit j of R_i and bit i of R_j
+                    row |= 1ull << (j - g0);
+                    atomicOr(R + j, 1ull << (e - g0));
+                }
+            }
+#pragma unroll
+            for (int o = G / 2; o >= 1; o >>= 1) row |= __shfl_xor_sync(0xffffffffu, row, o);
+            if (has && vl == 0 && row) atomicOr(R + e, row);
+        }
+    }
+    large = warp_sum(large);
+    if (lane == 0 && large) atomicAdd(ctrl + kLrLarge, large);
+}
+
+// thread per level-b entry of a small group: |L_{b+1}| and the count from the rows
+__global__ void k_lr_count(const uint2* __restrict__ lv, uint64_t nent, const uint64_t* __restrict__ cpos,
+                           uint64_t cw0, uint64_t cea, const unsigned long long* __restrict__ R,
+                           unsigned long long* __restrict__ ctrl) {
+    const uint64_t cbase = cpos[cea];
+    unsigned long long lvl = 0, cnt = 0;
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nent;
+         e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t p = lv[e].y;
+        const uint64_t g0 = cpos[p - cw0] - cbase, g1 = cpos[p - cw0 + 1] - cbase;
+        if (g1 - g0 > 64) continue;
+        const unsigned long long r = R[e];
+        lvl += __popcll(r);
+        for (unsigned long long b = r; b; b &= b - 1) cnt += __popcll(r & R[g0 + __ffsll((long long)b) - 1]);
+    }
+    lvl = warp_sum(lvl);
+    cnt = warp_sum(cnt);
+    if ((threadIdx.x & 31) == 0) {
+        if (lvl) atomicAdd(ctrl + kLrLevel, lvl);
+        add_u128(ctrl + kCountLo, cnt);
+    }
 }
 
 // ------------------------------------------------ SV intersection (ablation)

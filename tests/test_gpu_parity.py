@@ -543,3 +543,34 @@ def test_next2_binned_and_sv_variants(cuts, flag):
                 assert np.array_equal(_sorted_rows(c.enumerate("hybrid", cap_rows=want)), oracle.enumerate_rows(g, q))
             c.set_debug()
         c.close()
+
+
+def test_local_rows_and_pairs_on_clique_unions(cuts):
+    """The clique-tail paths (local 64-bit sibling rows, large-group fallback, pair-
+    shared last level) on K70 ∪ K30 ∪ ER: sibling groups of 68 (> 64, fallback) and
+    28 members (rows).  Every 5-vertex query Q has n!/(n-5)! embeddings in K_n, so
+    count = 70!/65! + 30!/25! + count in the ER part (oracle); level sizes likewise.
+    Default, CUTS_DEBUG_NO_LR and CUTS_DEBUG_NO_PAIRS must agree, at two arenas."""
+    from math import perm
+    er = er_graph(60, 200, 9)
+    edges = [(u, v) for u in range(70) for v in range(u + 1, 70)]
+    edges += [(70 + u, 70 + v) for u in range(30) for v in range(u + 1, 30)]
+    edges += [(100 + int(a), 100 + int(b)) for a, b in er.edge_list()]
+    g = graph_from_edges(160, edges)
+    for arena in (2 << 30, 96 << 20):
+        c = cuts(device=0, arena_bytes=arena)
+        c.load_csr(g)
+        for q in DENSE5[:3] + DENSE5[8:]:
+            qe, qlv = oracle.count(er, q, levels=True)
+            want = perm(70, 5) + perm(30, 5) + qe
+            order = oracle.order(q)
+            qd = q.degrees()
+            lv = [0] + [sum(perm(n, j) for n in (70, 30) if all(n - 1 >= qd[order[i]] for i in range(j))) + qlv[j]
+                        for j in range(1, 6)]
+            _set(c, q)
+            for flags in ({}, {"no_lr": True}, {"no_pairs": True}):
+                c.set_debug(**flags)
+                assert c.count("hybrid") == want, (arena, q.name, flags)
+                assert c.stats()["level_size"] == lv, (arena, q.name, flags)
+            c.set_debug()
+        c.close()

@@ -58,10 +58,11 @@ def main():
             c = ctx.count("hybrid")
             dt = time.time() - t
             st = ctx.stats()
-            deepest = max(st["level_size"][1:q.k])
+            stored = [j for j in range(1, q.k) if not (st["fused_levels"] >> j) & 1]
+            deepest = max(st["level_size"][j] for j in stored)
             rec = {"graph": spec.name, "gen_s": round(gen_s, 1), "query": q.name, "range": r, "roots": [rb, re],
                    "level1_canonical": l1, "count": c, "s": round(dt, 3), "emb_per_s": c / dt,
-                   "level_size": st["level_size"], "deepest_stored": deepest, "exceeds_180GB": 8 * deepest > 180e9,
+                   "level_size": st["level_size"], "deepest_stored": deepest, "stored_levels": stored, "exceeds_180GB": 8 * deepest > 180e9,
                    "chunks": st["chunks"], "windows": st["windows"], "launches": st["launches"],
                    "ms_extend": round(st["ms_extend"], 1), "ms_plan": round(st["ms_plan"], 1),
                    "peak_arena_bytes": st["peak_arena_bytes"], "debug": args.debug, "rep": rep}
