@@ -839,6 +839,13 @@ cuts_status lr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large) 
     const unsigned grid = (unsigned)std::min<uint64_t>((N + 255) / 256, (uint64_t)ctx->num_sms * 16);
     k_lr_count<<<grid, 256, 0, ctx->stream>>>(r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl);
     CK(cudaGetLastError());
+    {   // mid-size groups: a CTA each, adjacency in shared memory
+        static int occ = 0;
+        if (!occ) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_lr_group, 256, 0); if (occ < 1) occ = 1; }
+        CK(cudaMemsetAsync(ctx->ctrl + kLrWork, 0, sizeof(unsigned long long), ctx->stream));
+        k_lr_group<<<(unsigned)(ctx->num_sms * occ), 256, 0, ctx->stream>>>(r.g, r.t.lv[J], o.cpos, o.ea, o.eb, ctx->ctrl);
+        CK(cudaGetLastError());
+    }
     if (ctx->debug & CUTS_DEBUG_TIMING) {
         const int e1 = next_event(ctx);
         CK(cudaEventRecord(ctx->ev_pool[e1], ctx->stream));
@@ -848,7 +855,7 @@ cuts_status lr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large) 
     CK(cudaStreamSynchronize(ctx->stream));
     *large = ctx->h_ctrl[kLrLarge];
     ctx->st.chunks++;
-    ctx->st.launches += 2;
+    ctx->st.launches += 3;
     return CUTS_OK;
 }
 

@@ -21,6 +21,8 @@
 namespace cuts {
 
 constexpr int kMaxK = 8;
+constexpr int kLrMaxM = 512;                // local rows: largest sibling group held in shared memory
+constexpr int kLrWords = kLrMaxM / 32;
 constexpr int kTile = 256;   // items per CTA tile == threads per CTA
 
 struct QPlan {                 // query in matching-order positions
@@ -114,7 +116,7 @@ enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 // ancestor range, or the set-difference searches), reported beside the model
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
             kEnumCursor = 6, kNumSel = 7, kWork = 8, kBytesOut = 9, kBytesNeed = 10, kFind = 24,
-            kBins = 12, kLrLevel = 15, kLrLarge = 29, kDistLimbs = 56, kCtrlWords = 64 };
+            kBins = 12, kLrLevel = 15, kLrLarge = 29, kLrWork = 30, kDistLimbs = 56, kCtrlWords = 64 };
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
     if (v == 0) return;
@@ -317,7 +319,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         }
         if (ru.skip_small) {
             const uint64_t k0 = (uint64_t)idx - ru.w0;   // the parent is the ancestor (a = J-1)
-            if (ru.cpos[k0 + 1] - ru.cpos[k0] <= 64) {
+            if (ru.cpos[k0 + 1] - ru.cpos[k0] <= (uint64_t)kLrMaxM) {
                 ub[e] = 0;
                 src_off[e] = 0;
                 continue;
@@ -863,8 +865,8 @@ __global__ void __launch_bounds__(256, 6) k_lr_rows(Graph g, const uint2* __rest
                 v = x.x;
                 g0 = cpos[x.y - cw0] - cbase;
                 end = cpos[x.y - cw0 + 1] - cbase;
-                if (end - g0 > 64) {             // large group: the ordinary pipeline takes it
-                    if (vl == 0) large += 1;
+                if (end - g0 > 64) {             // k_lr_group or (> kLrMaxM) the ordinary pipeline
+                    if (vl == 0 && end - g0 > (uint64_t)kLrMaxM) large += 1;
                     has = false;
                 } else {
                     const uint32_t h = g.hub ? __ldg(g.hub + v) : kNoHub;
@@ -921,6 +923,98 @@ __global__ void __launch_bounds__(256, 6) k_lr_rows(Graph g, const uint2* __rest
     }
     large = warp_sum(large);
     if (lane == 0 && large) atomicAdd(ctrl + kLrLarge, large);
+}
+
+// Mid-size groups (64 < m <= kLrMaxM): one CTA per group builds the m x m sibling
+// adjacency in shared memory (each unordered pair tested once by a warp: hub bitmap or
+// cursor-narrowed binary search, both bits set), then the same bit algebra as
+// k_lr_count: |L_{b+1}| += popc(A_i), count += sum_{j in A_i} popc(A_i & A_j).
+// CTAs pull parent slots (groups) from a work counter.
+__global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restrict__ lv,
+                                                  const uint64_t* __restrict__ cpos, uint64_t cea, uint64_t ceb,
+                                                  unsigned long long* __restrict__ ctrl) {
+    __shared__ uint32_t S[kLrMaxM];
+    __shared__ uint32_t A[kLrMaxM][kLrWords];
+    __shared__ uint64_t s_q;
+    const uint64_t cbase = cpos[cea];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    unsigned long long lvl = 0, cnt = 0;
+    unsigned long long* work = ctrl + kLrWork;
+    for (;;) {
+        __syncthreads();
+        if (threadIdx.x == 0) s_q = cea + atomicAdd(work, 1ull);
+        __syncthreads();
+        const uint64_t q = s_q;
+        if (q >= ceb) break;
+        const uint64_t g0 = cpos[q] - cbase, g1 = cpos[q + 1] - cbase;
+        const uint32_t m = (uint32_t)(g1 - g0);
+        if (m <= 64 || m > (uint32_t)kLrMaxM) continue;          // uniform over the CTA
+        const uint32_t W = (m + 31) / 32;
+        for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) S[i] = lv[g0 + i].x;
+        for (uint32_t i = threadIdx.x; i < m * kLrWords; i += blockDim.x) (&A[0][0])[i] = 0u;
+        __syncthreads();
+        for (uint32_t i = warp; i + 1 < m; i += nw) {            // row i tests the members after it
+            const uint32_t v = S[i];
+            const uint32_t h = g.hub ? __ldg(g.hub + v) : kNoHub;
+            const uint32_t* lb;
+            uint32_t len = 0;
+            if (h != kNoHub) lb = g.bm + (uint64_t)h * g.words;
+            else { const uint64_t b = g.row_ptr[v]; lb = g.col + b; len = (uint32_t)(g.row_ptr[v + 1] - b); }
+            for (uint32_t j0 = i + 1; j0 < m; j0 += 32) {
+                const uint32_t j = j0 + lane;
+                const bool act = j < m;
+                const uint32_t c = act ? S[j] : 0u;
+                bool ok = false;
+                if (h != kNoHub) {
+                    ok = act && ((__ldg(lb + (c >> 5)) >> (c & 31)) & 1u);
+                } else {
+                    uint32_t pos = 0;
+                    if (act) {
+                        const uint32_t* b0 = lb;
+                        uint32_t l = len;
+                        while (l > 1) {
+                            const uint32_t half = l >> 1;
+                            b0 = (__ldg(b0 + half - 1) < c) ? b0 + half : b0;
+                            l -= half;
+                        }
+                        ok = len > 0 && __ldg(b0) == c;
+                        pos = (uint32_t)(b0 - lb);
+                    }
+                    const unsigned pw = __ballot_sync(0xffffffffu, act);
+                    const uint32_t mpos = __shfl_sync(0xffffffffu, pos, 31 - __clz(pw));
+                    lb += mpos;
+                    len -= mpos;
+                }
+                if (ok) {
+                    atomicOr(&A[i][j >> 5], 1u << (j & 31));
+                    atomicOr(&A[j][i >> 5], 1u << (i & 31));
+                }
+            }
+        }
+        __syncthreads();
+        for (uint32_t i = warp; i < m; i += nw) {                // bit algebra, a warp per row
+            uint32_t ri[kLrWords];
+#pragma unroll
+            for (int w = 0; w < kLrWords; ++w) ri[w] = (uint32_t)w < W ? A[i][w] : 0u;
+            if (lane == 0) {
+#pragma unroll
+                for (int w = 0; w < kLrWords; ++w) lvl += __popc(ri[w]);
+            }
+            for (uint32_t j = lane; j < m; j += 32) {             // lane takes the members j in row i
+                if (!((A[i][j >> 5] >> (j & 31)) & 1u)) continue;   // (smem: no dynamic register index)
+                uint32_t c = 0;
+#pragma unroll
+                for (int w = 0; w < kLrWords; ++w) c += (uint32_t)w < W ? __popc(ri[w] & A[j][w]) : 0u;
+                cnt += c;
+            }
+        }
+    }
+    lvl = warp_sum(lvl);
+    cnt = warp_sum(cnt);
+    if (lane == 0) {
+        if (lvl) atomicAdd(ctrl + kLrLevel, lvl);
+        add_u128(ctrl + kCountLo, cnt);
+    }
 }
 
 // thread per level-b entry of a small group: |L_{b+1}| and the count from the rows

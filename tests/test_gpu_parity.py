@@ -574,3 +574,28 @@ def test_local_rows_and_pairs_on_clique_unions(cuts):
                 assert c.stats()["level_size"] == lv, (arena, q.name, flags)
             c.set_debug()
         c.close()
+
+
+def test_local_rows_group_size_tiers(cuts):
+    """Sibling groups of every local-rows tier: two adjacent hubs over a circulant
+    C_600(1, 2) give the hub pair a group of 600 leaves (> 512: windowed fallback),
+    single hubs give mid-size groups (CTA-per-group shared-memory rows) and the
+    leaves small ones (64-bit rows).  Counts and level sizes == oracle, with and
+    without local rows."""
+    n = 600
+    edges = [(0, 1)] + [(h, 2 + i) for h in (0, 1) for i in range(n)]
+    edges += [(2 + i, 2 + (i + d) % n) for i in range(n) for d in (1, 2)]
+    edges += [(2 + n + i, 2 + (7 * i) % n) for i in range(100)]          # pendant vertices
+    g = graph_from_edges(2 + n + 100, edges)
+    c = cuts(device=0, arena_bytes=1 << 30)
+    c.load_csr(g)
+    cheap = ("K5", "K5-K2", "K5-P3", "K5-2K2", "K5-P4", "K5-K13", "K5-P3uK2", "K6", "K6-K2", "K6-P3")
+    for q in [q for q in DENSE5 + dense_family(6)[:3] if q.name in cheap]:   # oracle <= 2e7 embeddings each
+        want, lv = oracle.count(g, q, levels=True)
+        _set(c, q)
+        for flags in ({}, {"no_lr": True}):
+            c.set_debug(**flags)
+            assert c.count("hybrid") == want, (q.name, flags)
+            assert c.stats()["level_size"] == lv, (q.name, flags)
+        c.set_debug()
+    c.close()
