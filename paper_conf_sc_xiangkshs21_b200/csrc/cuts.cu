@@ -801,7 +801,7 @@ bool sym_last(const cuts_ctx* ctx, const Run& r, int J) {
 bool lr_level(const cuts_ctx* ctx, const Run& r, int J) {
     const int k = (int)ctx->q.k;
     if (J != k - 2 || J < 3 || r.enumerate || ctx->directed || !reuse_on(ctx, r)) return false;
-    if (ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED | CUTS_DEBUG_BYTES | CUTS_DEBUG_NO_LR)) return false;
+    if (ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED | CUTS_DEBUG_NO_LR)) return false;
     auto sym = [&](int L) {
         const uint32_t a = ctx->anc[L];
         return a && a + 1 == (uint32_t)L && (ctx->q.bw[L] & ~ctx->q.bw[a]) == (1u << a) && ctx->q.bwi[L] == 0 &&
@@ -822,28 +822,35 @@ cuts_status lr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large) 
     CK(cudaMemsetAsync(ctx->ctrl + kLrLarge, 0, sizeof(unsigned long long), ctx->stream));
     const double m = (double)N / (double)std::max<uint64_t>(o.eb - o.ea, 1);
     const double avg = m / 2;
+    const int cb = (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0;
     int e0 = -1;
     if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
     auto go = [&](auto kern, int G) {
-        static int occ[3] = {0, 0, 0};
-        int& oc = occ[G == 8 ? 0 : (G == 16 ? 1 : 2)];
+        static int occ[4] = {0, 0, 0, 0};
+        int& oc = occ[cb ? 3 : (G == 8 ? 0 : (G == 16 ? 1 : 2))];
         if (!oc) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&oc, kern, 256, 0); if (oc < 1) oc = 1; }
         const uint64_t grid = std::min<uint64_t>((uint64_t)ctx->num_sms * oc, (N * G + 255) / 256 + 1);
         const uint32_t batch = (uint32_t)std::min(256.0, std::max(2.0, 2048.0 / std::max(avg, 1.0) / (32 / G)));
         kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl, batch);
     };
-    if (avg >= 48) go(k_lr_rows<32>, 32);
-    else if (avg >= 12) go(k_lr_rows<16>, 16);
-    else go(k_lr_rows<8>, 8);
+    if (cb) go(k_lr_rows<16, true>, 16);
+    else if (avg >= 48) go(k_lr_rows<32, false>, 32);
+    else if (avg >= 12) go(k_lr_rows<16, false>, 16);
+    else go(k_lr_rows<8, false>, 8);
     CK(cudaGetLastError());
     const unsigned grid = (unsigned)std::min<uint64_t>((N + 255) / 256, (uint64_t)ctx->num_sms * 16);
-    k_lr_count<<<grid, 256, 0, ctx->stream>>>(r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl);
+    if (cb) k_lr_count<true><<<grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl, r.t,
+                                                           (uint32_t)J, ctx->q.bw[J], ctx->q.bw[J + 1]);
+    else k_lr_count<false><<<grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl, r.t,
+                                                          (uint32_t)J, ctx->q.bw[J], ctx->q.bw[J + 1]);
     CK(cudaGetLastError());
     {   // mid-size groups: a CTA each, adjacency in shared memory
         static int occ = 0;
-        if (!occ) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_lr_group, 256, 0); if (occ < 1) occ = 1; }
+        if (!occ) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_lr_group<false>, 256, 0); if (occ < 1) occ = 1; }
         CK(cudaMemsetAsync(ctx->ctrl + kLrWork, 0, sizeof(unsigned long long), ctx->stream));
-        k_lr_group<<<(unsigned)(ctx->num_sms * occ), 256, 0, ctx->stream>>>(r.g, r.t.lv[J], o.cpos, o.ea, o.eb, ctx->ctrl);
+        auto kg = cb ? k_lr_group<true> : k_lr_group<false>;
+        kg<<<(unsigned)(ctx->num_sms * occ), 256, 0, ctx->stream>>>(r.g, r.t.lv[J], o.cpos, o.ea, o.eb, ctx->ctrl, r.t,
+                                                                    (uint32_t)J, ctx->q.bw[J], ctx->q.bw[J + 1]);
         CK(cudaGetLastError());
     }
     if (ctx->debug & CUTS_DEBUG_TIMING) {
@@ -859,26 +866,29 @@ cuts_status lr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large) 
     return CUTS_OK;
 }
 
-// the whole level-J chunk in one k_pairs launch (no plan windows); CUTS_DEBUG_BYTES
-// runs take the windowed path instead, whose k_plan counts the §8.d model per entry
+// the whole level-J chunk in one k_pairs launch (no plan windows; with CUTS_DEBUG_BYTES
+// the kernel also counts the §8.d model of its entries)
 cuts_status pairs_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     const auto& o = ctx->ord[J - 1];
     const double m = (double)N / (double)std::max<uint64_t>(o.eb - o.ea, 1);   // siblings per group
     const double avg = m / 2;                                                  // tested per entry
+    const int cb = (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0;
     int e0 = -1;
     CK(cudaMemsetAsync(ctx->ctrl + kWork, 0, sizeof(unsigned long long), ctx->stream));
     if (ctx->debug & CUTS_DEBUG_TIMING) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
     auto go = [&](auto kern, int G) {
-        static int occ[3] = {0, 0, 0};
-        int& oc = occ[G == 8 ? 0 : (G == 16 ? 1 : 2)];
+        static int occ[4] = {0, 0, 0, 0};
+        int& oc = occ[cb ? 3 : (G == 8 ? 0 : (G == 16 ? 1 : 2))];
         if (!oc) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&oc, kern, 256, 0); if (oc < 1) oc = 1; }
         const uint64_t grid = std::min<uint64_t>((uint64_t)ctx->num_sms * oc, (N * G + 255) / 256 + 1);
         const uint32_t batch = (uint32_t)std::min(256.0, std::max(2.0, 2048.0 / std::max(avg, 1.0) / (32 / G)));
-        kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, ctx->ctrl, batch);
+        kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, ctx->ctrl, batch,
+                                                       r.t, (uint32_t)J, ctx->q.bw[J]);
     };
-    if (avg >= 48) go(k_pairs<32>, 32);
-    else if (avg >= 12) go(k_pairs<16>, 16);
-    else go(k_pairs<8>, 8);
+    if (cb) go(k_pairs<16, true>, 16);                   // instrumented (untimed) pass
+    else if (avg >= 48) go(k_pairs<32, false>, 32);
+    else if (avg >= 12) go(k_pairs<16, false>, 16);
+    else go(k_pairs<8, false>, 8);
     CK(cudaGetLastError());
     if (ctx->debug & CUTS_DEBUG_TIMING) {
         const int e1 = next_event(ctx);
@@ -894,7 +904,7 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     const int k = (int)ctx->q.k;
     const bool last = (J == k - 1);
     const uint64_t top_save = ctx->top;
-    if (last && !(ctx->debug & CUTS_DEBUG_BYTES) && sym_last(ctx, r, J)) return pairs_level(ctx, r, J, N);
+    if (last && sym_last(ctx, r, J)) return pairs_level(ctx, r, J, N);
     bool skip_small = false;
     if (lr_level(ctx, r, J) && free_bytes(ctx) >= N * 8 + (1u << 20)) {   // rows: 8 B per entry
         uint64_t large = 0;

@@ -728,6 +728,34 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
     }
 }
 
+// ------------------------------------- §8.d model bytes for the fused kernels
+// CUTS_DEBUG_BYTES in k_pairs / k_lr_*: the SURVEY §8.d per-entry model (DESIGN.md
+// §5) of the levels these kernels carry, so the instrumented pass runs the same
+// kernels as the timed one.  Degree sum of the lists of bw over the trie path of a
+// level-`lev` entry (walk `lev`-1 parent hops; path[lev-1] = the entry's vertex).
+__device__ __forceinline__ unsigned long long bw_degree_sum(const Graph& g, const Trie& t, uint32_t lev, uint64_t e,
+                                                            uint32_t bw) {
+    unsigned long long d = 0;
+    uint2 cur = t.lv[lev][e];
+    for (int p = (int)lev - 1; p >= 0; --p) {
+        if ((bw >> p) & 1u) d += __ldg(g.deg + cur.x);
+        if (p > 0) cur = t.lv[p][cur.y];
+    }
+    return d;
+}
+
+__device__ __forceinline__ void flush_model_bytes(unsigned long long plan, unsigned long long ext,
+                                                  unsigned long long out, unsigned long long need,
+                                                  unsigned long long* ctrl) {
+    plan = warp_sum(plan); ext = warp_sum(ext); out = warp_sum(out); need = warp_sum(need);
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(ctrl + kBytesPlan, plan);
+        atomicAdd(ctrl + kBytesExt, ext);
+        if (out) atomicAdd(ctrl + kBytesOut, out);
+        atomicAdd(ctrl + kBytesNeed, need);
+    }
+}
+
 // ------------------------------------------- symmetric last level: pair count
 // The count-only last level J = k-1 when the level J-1 -> J extension was written
 // ordered and the only condition left is adjacency to the entry itself (cliques;
@@ -742,11 +770,13 @@ __global__ void __launch_bounds__(256, (NL == 0 || (J <= 3 && NL < 2)) ? 6 : (J 
 //   lv     : the level-J chunk (.x = vertex, .y = index of the parent in level J-1)
 //   cpos   : level J-1 window's exclusive scan of child counts; cw0 = that window's
 //            start (parent index p -> slot p - cw0); cea = slot of the chunk's first parent
-template <int G>
+template <int G, bool count_bytes>
 __global__ void __launch_bounds__(256, 6) k_pairs(Graph g, const uint2* __restrict__ lv, uint64_t nent,
                                                   const uint64_t* __restrict__ cpos, uint64_t cw0, uint64_t cea,
-                                                  unsigned long long* __restrict__ ctrl, uint32_t batch) {
+                                                  unsigned long long* __restrict__ ctrl, uint32_t batch,
+                                                  Trie t, uint32_t lev, uint32_t bw) {
     const uint64_t cbase = cpos[cea];
+    unsigned long long b_plan = 0, b_ext = 0, b_need = 0;
     constexpr int VPW = 32 / G;
     constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
     const int lane = threadIdx.x & 31;
@@ -788,11 +818,17 @@ __global__ void __launch_bounds__(256, 6) k_pairs(Graph g, const uint2* __restri
 #pragma unroll
                 for (int o = 16; o >= G; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
             }
+            if (count_bytes && has && vl == 0) {   // model: entry + hops + bounds + every backward list
+                b_plan += 8ull + 8ull * (lev - 1) + 16ull * __popc(bw);
+                b_ext += 4ull * bw_degree_sum(g, t, lev, e, bw);
+                b_need += 8ull + 8ull + (bmp ? 4ull : 16ull);
+            }
             for (uint32_t it = 0; it < nit_max; ++it) {
                 const uint64_t j = e + 1 + (uint64_t)it * G + vl;
                 const bool act = has && j < end;
                 const uint32_t c = act ? lv[j].x : 0u;
                 bool ok = act;
+                if (count_bytes && act) b_need += 4ull + 4ull * (bmp ? 1u : (32u - __clz(len)));
                 if (bmp && act) ok = (__ldg(lb + (c >> 5)) >> (c & 31)) & 1u;   // hub: one bitmap probe
                 const bool pend = act && !bmp;
                 const unsigned pw = __ballot_sync(0xffffffffu, pend);
@@ -819,6 +855,8 @@ __global__ void __launch_bounds__(256, 6) k_pairs(Graph g, const uint2* __restri
     }
     my_count = warp_sum(my_count) * 2ull;          // every unordered pair counted once
     if (lane == 0) add_u128(ctrl + kCountLo, my_count);
+    // model: 4 B per intersection survivor = per child counted (both ends of each pair)
+    if (count_bytes) flush_model_bytes(b_plan, b_ext + (lane == 0 ? 4ull * my_count : 0ull), 0ull, b_need, ctrl);
 }
 
 // ------------------------------------------------ local rows (clique tail)
@@ -833,11 +871,12 @@ __global__ void __launch_bounds__(256, 6) k_pairs(Graph g, const uint2* __restri
 // k_lr_rows tests every unordered sibling pair once (hub bitmap or cursor-narrowed
 // binary search, as k_pairs) and sets both bits; k_lr_count does the bit algebra.
 // Groups with m > 64 are left to the ordinary pipeline (Reuse::skip_small).
-template <int G>
+template <int G, bool count_bytes>
 __global__ void __launch_bounds__(256, 6) k_lr_rows(Graph g, const uint2* __restrict__ lv, uint64_t nent,
                                                     const uint64_t* __restrict__ cpos, uint64_t cw0, uint64_t cea,
                                                     unsigned long long* __restrict__ R,
                                                     unsigned long long* __restrict__ ctrl, uint32_t batch) {
+    unsigned long long b_need = 0;
     constexpr int VPW = 32 / G;
     constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
     const uint64_t cbase = cpos[cea];
@@ -887,11 +926,13 @@ __global__ void __launch_bounds__(256, 6) k_lr_rows(Graph g, const uint2* __rest
                 for (int o = 16; o >= G; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
             }
             unsigned long long row = 0;
+            if (count_bytes && has && vl == 0) b_need += 8ull + 8ull + (bmp ? 4ull : 16ull) + 8ull;   // + the row
             for (uint32_t it = 0; it < nit_max; ++it) {
                 const uint64_t j = e + 1 + (uint64_t)it * G + vl;
                 const bool act = has && j < end;
                 const uint32_t c = act ? lv[j].x : 0u;
                 bool ok = act;
+                if (count_bytes && act) b_need += 4ull + 4ull * (bmp ? 1u : (32u - __clz(len)));
                 if (bmp && act) ok = (__ldg(lb + (c >> 5)) >> (c & 31)) & 1u;
                 const bool pend = act && !bmp;
                 const unsigned pw = __ballot_sync(0xffffffffu, pend);
@@ -923,6 +964,7 @@ __global__ void __launch_bounds__(256, 6) k_lr_rows(Graph g, const uint2* __rest
     }
     large = warp_sum(large);
     if (lane == 0 && large) atomicAdd(ctrl + kLrLarge, large);
+    if (count_bytes) flush_model_bytes(0, 0, 0, b_need, ctrl);
 }
 
 // Mid-size groups (64 < m <= kLrMaxM): one CTA per group builds the m x m sibling
@@ -930,12 +972,15 @@ __global__ void __launch_bounds__(256, 6) k_lr_rows(Graph g, const uint2* __rest
 // cursor-narrowed binary search, both bits set), then the same bit algebra as
 // k_lr_count: |L_{b+1}| += popc(A_i), count += sum_{j in A_i} popc(A_i & A_j).
 // CTAs pull parent slots (groups) from a work counter.
+template <bool count_bytes>
 __global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restrict__ lv,
                                                   const uint64_t* __restrict__ cpos, uint64_t cea, uint64_t ceb,
-                                                  unsigned long long* __restrict__ ctrl) {
+                                                  unsigned long long* __restrict__ ctrl, Trie t, uint32_t lev,
+                                                  uint32_t bw_b, uint32_t bw_c) {
     __shared__ uint32_t S[kLrMaxM];
     __shared__ uint32_t A[kLrMaxM][kLrWords];
     __shared__ uint64_t s_q;
+    unsigned long long b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
     const uint64_t cbase = cpos[cea];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     unsigned long long lvl = 0, cnt = 0;
@@ -965,6 +1010,7 @@ __global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restri
                 const bool act = j < m;
                 const uint32_t c = act ? S[j] : 0u;
                 bool ok = false;
+                if (count_bytes && act) b_need += 4ull * (h != kNoHub ? 1u : (32u - __clz(len)));
                 if (h != kNoHub) {
                     ok = act && ((__ldg(lb + (c >> 5)) >> (c & 31)) & 1u);
                 } else {
@@ -996,9 +1042,19 @@ __global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restri
             uint32_t ri[kLrWords];
 #pragma unroll
             for (int w = 0; w < kLrWords; ++w) ri[w] = (uint32_t)w < W ? A[i][w] : 0u;
-            if (lane == 0) {
+            unsigned long long pi = 0;
 #pragma unroll
-                for (int w = 0; w < kLrWords; ++w) lvl += __popc(ri[w]);
+            for (int w = 0; w < kLrWords; ++w) pi += __popc(ri[w]);
+            if (lane == 0) lvl += pi;
+            unsigned long long db = 0;
+            if (count_bytes) {        // the members share the parent's path: walk from member i
+                db = bw_degree_sum(g, t, lev, g0 + i, bw_b);
+                if (lane == 0) {
+                    b_plan += 8ull + 8ull * (lev - 1) + 16ull * __popc(bw_b) + pi * (8ull + 8ull * lev + 16ull * __popc(bw_c));
+                    b_ext += 4ull * db + 4ull * pi;
+                    b_out += 8ull * pi;
+                    b_need += 8ull + 8ull + 16ull;
+                }
             }
             for (uint32_t j = lane; j < m; j += 32) {             // lane takes the members j in row i
                 if (!((A[i][j >> 5] >> (j & 31)) & 1u)) continue;   // (smem: no dynamic register index)
@@ -1006,6 +1062,7 @@ __global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restri
 #pragma unroll
                 for (int w = 0; w < kLrWords; ++w) c += (uint32_t)w < W ? __popc(ri[w] & A[j][w]) : 0u;
                 cnt += c;
+                if (count_bytes) b_ext += 4ull * (db + __ldg(g.deg + S[j])) + 4ull * c;
             }
         }
     }
@@ -1015,14 +1072,20 @@ __global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restri
         if (lvl) atomicAdd(ctrl + kLrLevel, lvl);
         add_u128(ctrl + kCountLo, cnt);
     }
+    if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
 }
 
 // thread per level-b entry of a small group: |L_{b+1}| and the count from the rows
-__global__ void k_lr_count(const uint2* __restrict__ lv, uint64_t nent, const uint64_t* __restrict__ cpos,
+// With count_bytes it also adds the §8.d model of both carried levels: the level-b
+// entry's extension (lists of bw_b, survivors, children written) and every child's
+// count-only extension (lists of bw_b plus the child's own, survivors).
+template <bool count_bytes>
+__global__ void k_lr_count(Graph g, const uint2* __restrict__ lv, uint64_t nent, const uint64_t* __restrict__ cpos,
                            uint64_t cw0, uint64_t cea, const unsigned long long* __restrict__ R,
-                           unsigned long long* __restrict__ ctrl) {
+                           unsigned long long* __restrict__ ctrl, Trie t, uint32_t lev, uint32_t bw_b,
+                           uint32_t bw_c) {
     const uint64_t cbase = cpos[cea];
-    unsigned long long lvl = 0, cnt = 0;
+    unsigned long long lvl = 0, cnt = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
     for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nent;
          e += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t p = lv[e].y;
@@ -1030,7 +1093,24 @@ __global__ void k_lr_count(const uint2* __restrict__ lv, uint64_t nent, const ui
         if (g1 - g0 > 64) continue;
         const unsigned long long r = R[e];
         lvl += __popcll(r);
-        for (unsigned long long b = r; b; b &= b - 1) cnt += __popcll(r & R[g0 + __ffsll((long long)b) - 1]);
+        unsigned long long db = 0;
+        if (count_bytes) {
+            db = bw_degree_sum(g, t, lev, e, bw_b);
+            b_plan += 8ull + 8ull * (lev - 1) + 16ull * __popc(bw_b) +
+                      (unsigned long long)__popcll(r) * (8ull + 8ull * lev + 16ull * __popc(bw_c));
+            b_ext += 4ull * db + 4ull * __popcll(r);
+            b_out += 8ull * __popcll(r);
+            b_need += 8ull + 8ull + 16ull + 8ull;
+        }
+        for (unsigned long long b = r; b; b &= b - 1) {
+            const uint64_t j = g0 + __ffsll((long long)b) - 1;
+            const unsigned long long s2 = __popcll(r & R[j]);
+            cnt += s2;
+            if (count_bytes) {
+                b_ext += 4ull * (db + __ldg(g.deg + lv[j].x)) + 4ull * s2;
+                b_need += 8ull;
+            }
+        }
     }
     lvl = warp_sum(lvl);
     cnt = warp_sum(cnt);
@@ -1038,6 +1118,7 @@ __global__ void k_lr_count(const uint2* __restrict__ lv, uint64_t nent, const ui
         if (lvl) atomicAdd(ctrl + kLrLevel, lvl);
         add_u128(ctrl + kCountLo, cnt);
     }
+    if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
 }
 
 // ------------------------------------------------ SV intersection (ablation)

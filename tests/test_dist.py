@@ -129,10 +129,10 @@ def test_gloo_work_sharing_donations(world):
 
 
 def test_workload_root_ranges():
-    """The stated root range of C4 (absolute canonical positions [13500, 14000),
+    """The stated root range of C4 (absolute canonical positions [13500, 14400),
     clamped to the list) and the full range of the other configs."""
     from workloads import WORKLOADS, Workload
-    assert WORKLOADS["C4"].roots(1834382) == (13500, 14000)
+    assert WORKLOADS["C4"].roots(1834382) == (13500, 14400)
     assert WORKLOADS["C4"].roots(13600) == (13500, 13600)
     assert WORKLOADS["C4"].min_trie_bytes == 180e9
     assert Workload("x", "", (), root_range=(0, 1, 16)).roots(1600) == (0, 100)

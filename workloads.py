@@ -91,19 +91,19 @@ C3 = Workload(
 
 # configs[3]: 8-vertex dense query on R-MAT scale 22 forcing hybrid BFS/DFS chunking
 # beyond 180 GB: K8 on R-MAT(22, 16, .50, .20, .20) (n 4,194,304, 66.9 M edges, CSR
-# 547 MB), restricted to the stated canonical level-1 positions [13500, 14000) of
+# 547 MB), restricted to the stated canonical level-1 positions [13500, 14400) of
 # 1,834,382 (SURVEY §8.d allows a stated root range).  Calibrated in round 2
-# (profiles/r02b_c4sweep.jsonl): work is concentrated on the hub roots (tiers of
-# degree ~45 K, ~21 K, ~9.4 K, ~4 K); this range holds one ~9.4 K-degree hub
-# (position 13997) plus 499 ordinary roots: levels 9.1e3 / 4.0e5 / 8.3e6 / 1.7e8 /
-# 3.1e9 / 5.2e10 (the deepest stored level alone = 415 GB of 8 B trie entries, so
-# BFS cannot hold it and HYBRID chunking is on the timed path) and 8.0e11
-# embeddings per step.  The round-1 range [0, 1/16) holds two ~21 K hubs and took
-# 1,604 s per pass — too long for a 25-step driver run.
+# (profiles/r02b_c4_calibration.jsonl, r02g): the work sits on the hub roots
+# (degree tiers ~45 K, ~21 K, ~9.4 K, ~4 K); this range holds one ~21 K hub
+# (position 14341) and one ~9.4 K hub (13997) among 900 roots.  Levels 9.1e4 /
+# 2.2e6 / 5.6e7 / 1.5e9 / 3.8e10 / 9.1e11, count 2.02e13: the stored level 6 alone
+# is 304 GB of 8 B trie entries (level 7, 7.3 TB, is never stored), so it is cut
+# into DFS chunks.  The round-1 range [0, 1/16) holds two ~21 K hubs (1,604 s/pass
+# on the round-1 kernel).
 C4_GRAPH = GraphSpec("rmat_t", (22, 16, 0.50, 0.20, 0.20, 1))
 C4 = Workload(
-    "C4", "K8 on R-MAT(22,16,.50,.20,.20), canonical roots [13500, 14000) (one ~9.4K-degree hub); "
-          "hybrid count, deepest stored level > 180 GB",
-    ((C4_GRAPH, (dense_family(8)[0],)),), root_range=(13500, 14000, 0), min_trie_bytes=180e9)
+    "C4", "K8 on R-MAT(22,16,.50,.20,.20), canonical roots [13500, 14400) (a ~21K- and a ~9.4K-degree hub); "
+          "hybrid count, stored level > 180 GB",
+    ((C4_GRAPH, (dense_family(8)[0],)),), root_range=(13500, 14400, 0), min_trie_bytes=180e9)
 
 WORKLOADS = {"C1": C1, "C2": C2, "C3": C3, "C4": C4}
