@@ -28,6 +28,10 @@ for st in "$@"; do
     ncu_full) IFS=: read -r rx skip rest <<< "$arg"
              timeout -k 10 1800 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k "regex:${rx}" -s ${skip:-0} -c 1 \
              -o gpurun_out/${tag}_full -f $rest > gpurun_out/${tag}_ncu_full.log 2>&1; tail -5 gpurun_out/${tag}_ncu_full.log ;;
+    sanitize) for tool in ${arg:-memcheck racecheck synccheck}; do
+               timeout -k 10 1200 compute-sanitizer --tool $tool --error-exitcode 9 \
+                 python tools/sanitize_run.py > gpurun_out/${tag}_sanitize_${tool}.log 2>&1
+               echo "sanitize $tool rc=$?"; tail -4 gpurun_out/${tag}_sanitize_${tool}.log; done ;;
     *) echo "unknown step $name" ;;
   esac
   echo "== $tag $st rc=$? $(( $(date +%s) - t0 )) s"
