@@ -135,6 +135,13 @@ typedef struct {
                                   clique-like tail go through the trie pipeline (ordered
                                   write of level k-1, pair count) instead of 64-bit sibling
                                   adjacency rows of the level-(k-2) groups                  */
+#define CUTS_DEBUG_NO_DLR 4096u /* ablation: no deep local rows — the last three levels of a
+                                  clique-like count go through the ordered level-(k-3)
+                                  extension and the (k-2)-level local rows instead of the
+                                  level-(k-3) sibling rows carrying all three              */
+#define CUTS_DEBUG_GROUPS 2048u /* instrumentation: histogram of sibling-group sizes (children
+                                  per entry) of every ordered level, read with
+                                  cuts_debug_group_hist                                     */
 
 /* Create a context bound to opts->device / opts->stream / opts->arena.
  * CUTS_EINVAL if out/opts is NULL, arena is NULL or misaligned, or arena_bytes < 64 KiB. */
@@ -242,6 +249,14 @@ cuts_status cuts_get_stats(const cuts_ctx* ctx, cuts_stats* out);
 
 /* Instrumentation flags (CUTS_DEBUG_*); 0 for the timed product path. */
 cuts_status cuts_set_debug(cuts_ctx* ctx, uint32_t flags);
+
+/* CUTS_DEBUG_GROUPS result of the last count: out[(j * 16 + b) * 3 + {0, 1, 2}] =
+ * number of level-j sibling groups (the children of one level-(j-1) entry, written
+ * ordered) with size m in bucket b (b = 0: m = 0; b >= 1: 2^(b-1) <= m < 2^b, b = 15
+ * holds m >= 2^14), their sum of m, and their sum of m^2; j = 0..8.  out: HOST
+ * array of CUTS_GROUP_HIST_WORDS u64.  Zeros when the flag was off. */
+#define CUTS_GROUP_HIST_WORDS 432
+cuts_status cuts_debug_group_hist(cuts_ctx* ctx, uint64_t* out);
 
 /* Seed the search with flat prefixes instead of level 1 (the receiving side of
  * the dynamic redistribution of Alg. 3, P:1110-1144 l.16-20, "adjust depth",

@@ -269,14 +269,27 @@ class Cuts:
     def set_debug(self, timing: bool = False, bytes_: bool = False, no_reuse: bool = False,
                   no_pack: bool = False, first_source: bool = False, no_fast_count: bool = False,
                   preload_count: bool = False, binned: bool = False, sv: bool = False, no_pairs: bool = False,
-                  no_lr: bool = False):
+                  no_lr: bool = False, groups: bool = False, no_dlr: bool = False):
         """CUTS_DEBUG_* flags: instrumentation and the NEXT-2 ablations (include/cuts.h)."""
         flags = ((1 if timing else 0) | (2 if bytes_ else 0) | (4 if no_reuse else 0) |
                  (8 if no_pack else 0) | (16 if first_source else 0) | (32 if no_fast_count else 0) |
                  (64 if preload_count else 0) | (128 if binned else 0) | (256 if sv else 0) |
-                 (512 if no_pairs else 0) | (1024 if no_lr else 0))
+                 (512 if no_pairs else 0) | (1024 if no_lr else 0) | (2048 if groups else 0) |
+                 (4096 if no_dlr else 0))
         self._check(self.lib.cuts_set_debug(self.h, flags))
         return self
+
+    def group_hist(self) -> dict:
+        """CUTS_DEBUG_GROUPS: {level: [(bucket, groups, sum m, sum m^2), ...]} of the last count."""
+        buf = (ctypes.c_uint64 * L.GROUP_HIST_WORDS)()
+        self._check(self.lib.cuts_debug_group_hist(self.h, buf))
+        out = {}
+        for j in range(9):
+            rows = [(b, buf[(j * 16 + b) * 3], buf[(j * 16 + b) * 3 + 1], buf[(j * 16 + b) * 3 + 2])
+                    for b in range(16) if buf[(j * 16 + b) * 3]]
+            if rows:
+                out[j] = rows
+        return out
 
     def count(self, mode="hybrid") -> int:
         """Exact count (Python int; values >= 2^64 are returned in full)."""

@@ -746,6 +746,11 @@ cuts_status hybrid_ordered(cuts_ctx* ctx, Run& r, int J, Window& w) {
     Window wa = w;
     wa.ord_cnt = w.ub;
     TRY(extend_range(ctx, r, J, wa, 0, w.total, kCount, nullptr, 0));
+    if (ctx->debug & CUTS_DEBUG_GROUPS) {
+        k_group_hist<<<std::min<uint32_t>((w.W + 255) / 256, 1024u), 256, 0, ctx->stream>>>(
+            w.ub, w.W, ctx->ctrl + kGroupHist + 48 * (J + 1));
+        CK(cudaGetLastError());
+    }
     CK(cub::DeviceScan::ExclusiveSum(w.cub_tmp, w.cub_bytes, w.ub, w.cpos, (int64_t)w.W + 1, ctx->stream));
     ctx->st.launches += 2;
     for (uint32_t ea = 0; ea < w.W;) {
@@ -866,6 +871,127 @@ cuts_status lr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large) 
     return CUTS_OK;
 }
 
+// deep local rows: level J = k-3 of a clique-like tail whose last three
+// extensions only add adjacency to the newest vertex — the rows of the level-J sibling
+// groups write level J+1 (stored, chunked) and carry levels J+2 and the count
+bool dlr_level(const cuts_ctx* ctx, const Run& r, int J) {
+    const int k = (int)ctx->q.k;
+    if (J != k - 3 || J < 3 || r.enumerate || ctx->directed || !reuse_on(ctx, r)) return false;
+    if (ctx->debug & (CUTS_DEBUG_NO_PAIRS | CUTS_DEBUG_BINNED | CUTS_DEBUG_NO_LR | CUTS_DEBUG_NO_DLR)) return false;
+    auto sym = [&](int L) {
+        const uint32_t a = ctx->anc[L];
+        return a && a + 1 == (uint32_t)L && (ctx->q.bw[L] & ~ctx->q.bw[a]) == (1u << a) && ctx->q.bwi[L] == 0 &&
+               ctx->q.qdeg[L] <= ctx->q.qdeg[a];
+    };
+    return sym(J) && sym(J + 1) && sym(J + 2) && ctx->ord[J - 1].valid;
+}
+
+// rows of the level-J chunk's groups, then level J+1 in entry-aligned chunks that fit
+// the arena, each followed by the two-level tail; *large = entries left to the
+// windowed pipeline (groups of more than kDlrMaxM members)
+cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large, bool* applied) {
+    const auto& o = ctx->ord[J - 1];
+    const uint64_t ng = o.eb - o.ea;
+    const int cb = (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0;
+    const bool timing = (ctx->debug & CUTS_DEBUG_TIMING) != 0;
+    Dlr a{r.t.lv[J], N, o.cpos, o.w0, o.ea, o.eb, nullptr, nullptr};
+    size_t cub_bytes = 0;
+    const uint64_t nscan = std::max<uint64_t>(ng, N) + 1;
+    CK(cub::DeviceScan::ExclusiveSum(nullptr, cub_bytes, (uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)nscan, ctx->stream));
+    uint64_t off;
+    TRY(alloc_top(ctx, align_up((ng + 1) * 8) * 2 + align_up((N + 1) * 8) * 2 + align_up(cub_bytes), &off));
+    char* p = ctx->arena + off;
+    uint64_t* rw = (uint64_t*)p; p += align_up((ng + 1) * 8);
+    uint64_t* roff = (uint64_t*)p; p += align_up((ng + 1) * 8);
+    uint64_t* cnt = (uint64_t*)p; p += align_up((N + 1) * 8);
+    uint64_t* cposb = (uint64_t*)p; p += align_up((N + 1) * 8);
+    void* cub_tmp = p;
+    int e0 = -1;
+    if (timing) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
+    CK(cudaMemsetAsync(ctx->ctrl + kDlrLarge, 0, 2 * sizeof(unsigned long long), ctx->stream));   // + kDlrWork
+    const unsigned lg = (unsigned)std::min<uint64_t>((ng + 256) / 256, (uint64_t)ctx->num_sms * 8);
+    k_dlr_layout<<<lg, 256, 0, ctx->stream>>>(a, rw, ctx->ctrl);
+    CK(cudaGetLastError());
+    CK(cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, rw, roff, (int64_t)ng + 1, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_ctrl + kDlrLarge, ctx->ctrl + kDlrLarge, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 8, roff + ng, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    *large = ctx->h_ctrl[kDlrLarge];
+    const uint64_t words = ctx->h_ctrl[kCtrlWords + 8];
+    // the rows must leave room for level-(J+1) chunks of a useful size; else the lr path
+    *applied = words * 8 + (N + (1ull << 27)) * sizeof(uint2) <= free_bytes(ctx);
+    if (!*applied) return CUTS_OK;
+    TRY(alloc_top(ctx, std::max<uint64_t>(words, 1) * 8, &off));
+    a.R = (unsigned long long*)(ctx->arena + off);
+    a.roff = roff;
+    CK(cudaMemsetAsync(a.R, 0, words * 8, ctx->stream));
+    const double avg = (double)N / (double)std::max<uint64_t>(ng, 1) / 2;     // members tested per entry
+    auto go = [&](auto kern, int G) {
+        static int occ[4] = {0, 0, 0, 0};
+        int& oc = occ[cb ? 3 : (G == 8 ? 0 : (G == 16 ? 1 : 2))];
+        if (!oc) { cudaOccupancyMaxActiveBlocksPerMultiprocessor(&oc, kern, 256, 0); if (oc < 1) oc = 1; }
+        const uint64_t grid = std::min<uint64_t>((uint64_t)ctx->num_sms * oc, (N * G + 255) / 256 + 1);
+        const uint32_t batch = (uint32_t)std::min(256.0, std::max(2.0, 2048.0 / std::max(avg, 1.0) / (32 / G)));
+        kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, a, ctx->ctrl, batch);
+    };
+    if (cb) go(k_dlr_rows<16, true>, 16);
+    else if (avg >= 48) go(k_dlr_rows<32, false>, 32);
+    else if (avg >= 12) go(k_dlr_rows<16, false>, 16);
+    else go(k_dlr_rows<8, false>, 8);
+    CK(cudaGetLastError());
+    const unsigned gc = (unsigned)std::min<uint64_t>((N + 256) / 256, (uint64_t)ctx->num_sms * 16);
+    if (cb) k_dlr_counts<true><<<gc, 256, 0, ctx->stream>>>(r.g, r.t, a, cnt, ctx->ctrl, (uint32_t)J, ctx->q.bw[J]);
+    else k_dlr_counts<false><<<gc, 256, 0, ctx->stream>>>(r.g, r.t, a, cnt, ctx->ctrl, (uint32_t)J, ctx->q.bw[J]);
+    CK(cudaGetLastError());
+    CK(cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, cnt, cposb, (int64_t)N + 1, ctx->stream));
+    ctx->st.launches += 6;
+    if (timing) {
+        const int e1 = next_event(ctx);
+        CK(cudaEventRecord(ctx->ev_pool[e1], ctx->stream));
+        ctx->ev_ext.push_back({e0, e1});
+    }
+    // level J+1 in entry-aligned chunks: write, then the two fused levels
+    for (uint64_t ea = 0; ea < N;) {
+        uint64_t cap;
+        TRY(chunk_cap(ctx, J, &cap));
+        k_find_chunk<<<1, 1, 0, ctx->stream>>>(cposb, cposb, (uint32_t)N, (uint32_t)ea, cap, ctx->ctrl + kFind);
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(ctx->h_ctrl + kFind, ctx->ctrl + kFind, 2 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        ctx->st.launches++;
+        const uint64_t eb = ctx->h_ctrl[kFind], size = ctx->h_ctrl[kFind + 1];
+        if (eb <= ea) return fail(ctx, CUTS_ENOMEM, "HYBRID: one level-%d entry's children exceed the arena share", J);
+        if (size) {
+            const uint64_t bot_save = ctx->bot;
+            TRY(alloc_bot(ctx, size * sizeof(uint2), &off));
+            uint2* out = (uint2*)(ctx->arena + off);
+            int t0 = -1;
+            if (timing) { t0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[t0], ctx->stream)); }
+            const unsigned gw = (unsigned)std::min<uint64_t>((eb - ea + 255) / 256, (uint64_t)ctx->num_sms * 16);
+            k_dlr_write<<<gw, 256, 0, ctx->stream>>>(a, cposb, ea, eb, out);
+            CK(cudaGetLastError());
+            r.t.lv[J + 1] = out;
+            const unsigned gt = (unsigned)std::min<uint64_t>((size + 255) / 256, (uint64_t)ctx->num_sms * 16);
+            if (cb) k_dlr_tail<true><<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
+                                                                (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            else k_dlr_tail<false><<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
+                                                                (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            CK(cudaGetLastError());
+            if (timing) {
+                const int t1 = next_event(ctx);
+                CK(cudaEventRecord(ctx->ev_pool[t1], ctx->stream));
+                ctx->ev_ext.push_back({t0, t1});
+            }
+            ctx->st.level_size[J + 1] += size;
+            ctx->st.chunks++;
+            ctx->st.launches += 2;
+            ctx->bot = bot_save;
+        }
+        ea = eb;
+    }
+    return CUTS_OK;
+}
+
 // the whole level-J chunk in one k_pairs launch (no plan windows; with CUTS_DEBUG_BYTES
 // the kernel also counts the §8.d model of its entries)
 cuts_status pairs_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
@@ -905,14 +1031,26 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     const bool last = (J == k - 1);
     const uint64_t top_save = ctx->top;
     if (last && sym_last(ctx, r, J)) return pairs_level(ctx, r, J, N);
-    bool skip_small = false;
-    if (lr_level(ctx, r, J) && free_bytes(ctx) >= N * 8 + (1u << 20)) {   // rows: 8 B per entry
+    uint32_t skip_small = 0;
+    bool dlr = false;
+    if (dlr_level(ctx, r, J) && free_bytes(ctx) >= N * 32 + (64ull << 20)) {   // the two scans + room
+        uint64_t large = 0;
+        TRY(dlr_chunk(ctx, r, J, N, &large, &dlr));
+        ctx->top = top_save;
+        if (dlr) {
+            ctx->st.fused_levels |= 1ull << (J + 2);   // level k-1 of these groups is never stored
+            if (large == 0) return CUTS_OK;
+            skip_small = (uint32_t)kDlrMaxM;
+        }
+    }
+    if (dlr) {
+    } else if (lr_level(ctx, r, J) && free_bytes(ctx) >= N * 8 + (1u << 20)) {   // rows: 8 B per entry
         uint64_t large = 0;
         TRY(lr_chunk(ctx, r, J, N, &large));
         ctx->top = top_save;
         ctx->st.fused_levels |= 1ull << (J + 1);   // level k-1 of the small groups is never stored
         if (large == 0) return CUTS_OK;       // every group was small: nothing left at this level
-        skip_small = true;
+        skip_small = (uint32_t)kLrMaxM;
     }
     const bool ordered = !last && reuse_on(ctx, r) && ((ctx->need_ord >> J) & 1u);
     ctx->dfs_on[J] = true;
@@ -929,7 +1067,7 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
         const uint32_t a = ctx->anc[J];
         if (a && reuse_on(ctx, r) && ctx->ord[a].valid)
             w.ru = Reuse{ctx->ord[a].lv, ctx->ord[a].cpos, ctx->ord[a].w0, ctx->ord[a].ea, a, ctx->q.bw[a],
-                         sym_last(ctx, r, J) ? 1u : 0u, skip_small ? 1u : 0u};
+                         sym_last(ctx, r, J) ? 1u : 0u, skip_small};
         TRY(alloc_window(ctx, J, w.W, &w));
         TRY(plan_window(ctx, r, J, w));
         if (last) {
@@ -1196,6 +1334,8 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     ctx->top = ctx->arena_bytes & ~(kAlign - 1);
     ctx->peak = ctx->bot;
     CK(cudaMemsetAsync(ctx->ctrl, 0, kCtrlWords * sizeof(unsigned long long), ctx->stream));
+    if (ctx->debug & CUTS_DEBUG_GROUPS)
+        CK(cudaMemsetAsync(ctx->ctrl + kGroupHist, 0, kGroupHistWords * sizeof(unsigned long long), ctx->stream));
     if (ctx->debug & CUTS_DEBUG_PRELOAD_COUNT) {   // test hook: the 128-bit carry and CUTS_EOVERFLOW
         ctx->h_ctrl[kCtrlWords + 16] = kPreloadCount;
         CK(cudaMemcpyAsync(ctx->ctrl + kCountLo, ctx->h_ctrl + kCtrlWords + 16, 8, cudaMemcpyHostToDevice, ctx->stream));
@@ -1564,6 +1704,15 @@ cuts_status cuts_get_stats(const cuts_ctx* ctx, cuts_stats* out) {
 cuts_status cuts_set_debug(cuts_ctx* ctx, uint32_t flags) {
     if (!ctx) return CUTS_EINVAL;
     ctx->debug = flags;
+    return CUTS_OK;
+}
+
+cuts_status cuts_debug_group_hist(cuts_ctx* ctx, uint64_t* out) {
+    if (!ctx || !out) return CUTS_EINVAL;
+    CK(cudaSetDevice(ctx->device));
+    CK(cudaMemcpyAsync(out, ctx->ctrl + kGroupHist, kGroupHistWords * sizeof(unsigned long long),
+                       cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
     return CUTS_OK;
 }
 

@@ -23,6 +23,8 @@ namespace cuts {
 constexpr int kMaxK = 8;
 constexpr int kLrMaxM = 512;                // local rows: largest sibling group held in shared memory
 constexpr int kLrWords = kLrMaxM / 32;
+constexpr int kLrBatch = 256;
+constexpr int kDlrMaxM = 1024;             // deep local rows: largest sibling group (16 u64 words per row)              // k_lr_group: parent slots claimed per CTA fetch
 constexpr int kTile = 256;   // items per CTA tile == threads per CTA
 
 struct QPlan {                 // query in matching-order positions
@@ -78,8 +80,9 @@ struct Reuse {
     // siblings AFTER itself and the count-only kernel doubles its sum (every unordered
     // sibling pair tested once instead of twice)
     uint32_t sym;
-    // local rows took this level's small sibling groups (<= 64 members): k_plan gives
-    // their entries no candidates (ub = 0) so the windowed pipeline only sees the rest
+    // local rows took this level's sibling groups of <= skip_small members (0: none):
+    // k_plan gives their entries no candidates (ub = 0) so the windowed pipeline only
+    // sees the rest
     uint32_t skip_small;
 };
 
@@ -116,7 +119,8 @@ enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 // ancestor range, or the set-difference searches), reported beside the model
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
             kEnumCursor = 6, kNumSel = 7, kWork = 8, kBytesOut = 9, kBytesNeed = 10, kFind = 24,
-            kBins = 12, kLrLevel = 15, kLrLarge = 29, kLrWork = 30, kDistLimbs = 56, kCtrlWords = 64 };
+            kBins = 12, kLrLevel = 15, kLrLarge = 29, kLrWork = 30, kDlrLarge = 31, kDlrWork = 32, kDistLimbs = 56, kCtrlWords = 64,
+            kGroupHist = 64, kGroupHistWords = 432 };   // CUTS_DEBUG_GROUPS: [level][16 buckets][3]
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
     if (v == 0) return;
@@ -319,7 +323,7 @@ __global__ void __launch_bounds__(256) k_plan(Graph g, Trie t, QPlan q, uint64_t
         }
         if (ru.skip_small) {
             const uint64_t k0 = (uint64_t)idx - ru.w0;   // the parent is the ancestor (a = J-1)
-            if (ru.cpos[k0 + 1] - ru.cpos[k0] <= (uint64_t)kLrMaxM) {
+            if (ru.cpos[k0 + 1] - ru.cpos[k0] <= (uint64_t)ru.skip_small) {
                 ub[e] = 0;
                 src_off[e] = 0;
                 continue;
@@ -978,25 +982,39 @@ __global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restri
                                                   unsigned long long* __restrict__ ctrl, Trie t, uint32_t lev,
                                                   uint32_t bw_b, uint32_t bw_c) {
     __shared__ uint32_t S[kLrMaxM];
-    __shared__ uint32_t A[kLrMaxM][kLrWords];
+    __shared__ uint32_t A[kLrMaxM][kLrWords + 1];   // odd row stride: lanes on distinct rows hit distinct banks
     __shared__ uint64_t s_q;
+    __shared__ uint32_t s_n, s_list[kLrBatch];
     unsigned long long b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
     const uint64_t cbase = cpos[cea];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     unsigned long long lvl = 0, cnt = 0;
     unsigned long long* work = ctrl + kLrWork;
     for (;;) {
+        // a batch of kLrBatch parent slots per CTA: one thread tests each slot's group
+        // size (coalesced cpos reads) and the mid-size groups are listed in shared memory
         __syncthreads();
-        if (threadIdx.x == 0) s_q = cea + atomicAdd(work, 1ull);
+        if (threadIdx.x == 0) { s_q = cea + atomicAdd(work, (unsigned long long)kLrBatch); s_n = 0; }
         __syncthreads();
-        const uint64_t q = s_q;
-        if (q >= ceb) break;
+        const uint64_t qb = s_q;
+        if (qb >= ceb) break;
+        for (uint32_t x = threadIdx.x; x < (uint32_t)kLrBatch; x += blockDim.x) {
+            const uint64_t q = qb + x;
+            if (q < ceb) {
+                const uint64_t m = cpos[q + 1] - cpos[q];
+                if (m > 64 && m <= (uint64_t)kLrMaxM) s_list[atomicAdd(&s_n, 1u)] = x;
+            }
+        }
+        __syncthreads();
+        const uint32_t nlist = s_n;
+        for (uint32_t li = 0; li < nlist; ++li) {
+        __syncthreads();
+        const uint64_t q = qb + s_list[li];
         const uint64_t g0 = cpos[q] - cbase, g1 = cpos[q + 1] - cbase;
         const uint32_t m = (uint32_t)(g1 - g0);
-        if (m <= 64 || m > (uint32_t)kLrMaxM) continue;          // uniform over the CTA
         const uint32_t W = (m + 31) / 32;
         for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) S[i] = lv[g0 + i].x;
-        for (uint32_t i = threadIdx.x; i < m * kLrWords; i += blockDim.x) (&A[0][0])[i] = 0u;
+        for (uint32_t i = threadIdx.x; i < m * (kLrWords + 1); i += blockDim.x) (&A[0][0])[i] = 0u;
         __syncthreads();
         for (uint32_t i = warp; i + 1 < m; i += nw) {            // row i tests the members after it
             const uint32_t v = S[i];
@@ -1065,6 +1083,7 @@ __global__ void __launch_bounds__(256) k_lr_group(Graph g, const uint2* __restri
                 if (count_bytes) b_ext += 4ull * (db + __ldg(g.deg + S[j])) + 4ull * c;
             }
         }
+        }
     }
     lvl = warp_sum(lvl);
     cnt = warp_sum(cnt);
@@ -1119,6 +1138,311 @@ __global__ void k_lr_count(Graph g, const uint2* __restrict__ lv, uint64_t nent,
         add_u128(ctrl + kCountLo, cnt);
     }
     if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
+}
+
+// ------------------------------------------------ deep local rows (clique tail)
+// DESIGN.md §7 "deep local rows": the local-rows idea one level higher.  When the
+// last THREE extensions of a count-only query only add adjacency to the newest vertex
+// (Reuse::sym conditions at b, b+1, b+2 with b = k-3), a level-b sibling group
+// G = (G[0] < ... < G[m-1]) (the ordered children of one level-(b-1) entry) and its
+// adjacency rows A_t = {s : G[s] in N(G[t])} carry all three:
+//   children(e_t)            = G[A_t]                       -> level b+1, WRITTEN (trie)
+//   children((e_t, G[s]))    = G[A_t & A_s]                 -> |L_{b+2}| (fused)
+//   children((e_t, G[s], G[l])) = G[A_t & A_s & A_l]        -> the count
+// Rows are W = ceil(m/64) u64 words; every unordered pair of G is tested once (hub
+// bitmap or cursor-narrowed binary search), so a group costs m^2/2 membership tests
+// instead of the m_child^2/2 of every child group below it.  Groups of more than
+// kDlrMaxM members are left to the windowed pipeline (Reuse::skip_small).
+struct Dlr {
+    const uint2* lv;            // level-b chunk (.x vertex, .y parent index in level b-1)
+    uint64_t n;                 // entries of the chunk
+    const uint64_t* cpos;       // level b-1 window: exclusive scan of child counts
+    uint64_t w0, ea, eb;        // window start; parent slots [ea, eb) own the chunk (window-relative)
+    const uint64_t* roff;       // row word offset of each parent slot's group (slot - ea)
+    unsigned long long* R;      // rows
+};
+
+struct DlrGrp {
+    uint64_t g0;                // first member (chunk index)
+    uint64_t rb;                // first row word
+    uint32_t m, W;
+};
+
+__device__ __forceinline__ DlrGrp dlr_group(const Dlr& a, uint64_t e) {
+    const uint64_t q = (uint64_t)a.lv[e].y - a.w0;
+    const uint64_t c0 = a.cpos[q], c1 = a.cpos[q + 1];
+    DlrGrp gr;
+    gr.g0 = c0 - a.cpos[a.ea];
+    gr.m = (uint32_t)(c1 - c0);
+    gr.W = (gr.m + 63) / 64;
+    gr.rb = a.roff[q - a.ea];
+    return gr;
+}
+
+// per parent slot: row words of its group (0 when it is left to the windowed pipeline)
+__global__ void k_dlr_layout(Dlr a, uint64_t* __restrict__ rw, unsigned long long* __restrict__ ctrl) {
+    unsigned long long large = 0;
+    const uint64_t ng = a.eb - a.ea;
+    for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x <= ng; x += (uint64_t)gridDim.x * blockDim.x) {
+        if (x == ng) { rw[ng] = 0; continue; }
+        const uint64_t m = a.cpos[a.ea + x + 1] - a.cpos[a.ea + x];
+        rw[x] = m <= (uint64_t)kDlrMaxM ? m * ((m + 63) / 64) : 0ull;
+        if (m > (uint64_t)kDlrMaxM) large += m;
+    }
+    large = warp_sum(large);
+    if ((threadIdx.x & 31) == 0 && large) atomicAdd(ctrl + kDlrLarge, large);
+}
+
+// Rows: a virtual warp of G lanes per entry t tests the members after it, in G-aligned
+// blocks of the group so the block's ballot is one aligned G-bit piece of row t (one
+// atomicOr); each hit also sets bit t of the other member's row.
+template <int G, bool count_bytes>
+__global__ void __launch_bounds__(256, 6) k_dlr_rows(Graph g, Dlr a, unsigned long long* __restrict__ ctrl,
+                                                     uint32_t batch) {
+    unsigned long long b_need = 0;
+    constexpr int VPW = 32 / G;
+    constexpr unsigned kGMask = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
+    const int lane = threadIdx.x & 31;
+    const int vl = lane & (G - 1);
+    const int vb = lane & ~(G - 1);
+    unsigned long long* work = ctrl + kDlrWork;
+    uint32_t* R32 = (uint32_t*)a.R;
+    for (;;) {
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(work, (unsigned long long)VPW * batch);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (base >= a.n) break;
+#pragma unroll 1
+        for (uint32_t bt = 0; bt < batch; ++bt) {
+            const uint64_t e = base + (uint64_t)bt * VPW + (uint64_t)(lane / G);
+            if (!__any_sync(0xffffffffu, e < a.n)) break;
+            bool has = e < a.n;
+            uint32_t len = 0, te = 0, jb = 0, m = 0, W = 0;
+            uint64_t g0 = 0, rb = 0;
+            const uint32_t* lb = g.col;
+            bool bmp = false;
+            if (has) {
+                const DlrGrp gr = dlr_group(a, e);
+                g0 = gr.g0; m = gr.m; W = gr.W; rb = gr.rb;
+                te = (uint32_t)(e - g0);
+                has = m >= 2 && m <= (uint32_t)kDlrMaxM && te + 1 < m;
+                if (has) {
+                    jb = (te + 1) & ~(uint32_t)(G - 1);
+                    const uint32_t v = a.lv[e].x;
+                    const uint32_t h = g.hub ? __ldg(g.hub + v) : kNoHub;
+                    if (h != kNoHub) {
+                        bmp = true;
+                        lb = g.bm + (uint64_t)h * g.words;
+                    } else {
+                        const uint64_t b = g.row_ptr[v];
+                        lb = g.col + b;
+                        len = (uint32_t)(g.row_ptr[v + 1] - b);
+                    }
+                }
+            }
+            const uint32_t nit = has ? (m - jb + G - 1) / G : 0u;
+            uint32_t nit_max = nit;
+            if (VPW > 1) {
+#pragma unroll
+                for (int o = 16; o >= G; o >>= 1) nit_max = max(nit_max, __shfl_xor_sync(0xffffffffu, nit_max, o));
+            }
+            if (count_bytes && has && vl == 0) b_need += 8ull + 16ull + (bmp ? 4ull : 16ull);
+            uint32_t* row_e = R32 + 2 * (rb + (uint64_t)te * W);
+            for (uint32_t it = 0; it < nit_max; ++it) {
+                const uint32_t jj = jb + it * G + vl;
+                const bool act = has && jj > te && jj < m;
+                const uint32_t c = act ? a.lv[g0 + jj].x : 0u;
+                bool ok = act;
+                if (count_bytes && act) b_need += 4ull + 4ull * (bmp ? 1u : (32u - __clz(len)));
+                if (bmp && act) ok = (__ldg(lb + (c >> 5)) >> (c & 31)) & 1u;
+                const bool pend = act && !bmp;
+                const unsigned pw = __ballot_sync(0xffffffffu, pend);
+                uint32_t pos = 0;
+                if (pend) {
+                    const uint32_t* b0 = lb;
+                    uint32_t l = len;
+                    while (l > 1) {
+                        const uint32_t half = l >> 1;
+                        b0 = (__ldg(b0 + half - 1) < c) ? b0 + half : b0;
+                        l -= half;
+                    }
+                    ok = len > 0 && __ldg(b0) == c;
+                    pos = (uint32_t)(b0 - lb);
+                }
+                const unsigned pv = (pw >> vb) & kGMask;
+                const int hl = pv ? vb + 31 - __clz(pv) : lane;
+                const uint32_t mpos = __shfl_sync(0xffffffffu, pos, hl);
+                if (pv) { lb += mpos; len -= mpos; }
+                const unsigned seg = (__ballot_sync(0xffffffffu, ok) >> vb) & kGMask;
+                if (ok) atomicOr(R32 + 2 * (rb + (uint64_t)jj * W) + (te >> 5), 1u << (te & 31));
+                if (vl == 0 && seg) {
+                    const uint32_t j0 = jb + it * G;
+                    atomicOr(row_e + (j0 >> 5), seg << (j0 & 31));
+                }
+            }
+        }
+    }
+    if (count_bytes) flush_model_bytes(0, 0, 0, b_need, ctrl);
+}
+
+// children per entry (0 outside the eligible groups); with count_bytes the §8.d model
+// of the level-b -> b+1 extension these rows stand for
+template <bool count_bytes>
+__global__ void k_dlr_counts(Graph g, Trie t, Dlr a, uint64_t* __restrict__ cnt, unsigned long long* __restrict__ ctrl,
+                             uint32_t lev, uint32_t bw_b) {
+    unsigned long long b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e <= a.n; e += (uint64_t)gridDim.x * blockDim.x) {
+        if (e == a.n) { cnt[e] = 0; continue; }
+        const DlrGrp gr = dlr_group(a, e);
+        uint64_t c = 0;
+        if (gr.m <= (uint32_t)kDlrMaxM) {
+            const unsigned long long* r = a.R + gr.rb + (e - gr.g0) * gr.W;
+            for (uint32_t w = 0; w < gr.W; ++w) c += __popcll(r[w]);
+            if (count_bytes) {
+                b_plan += 8ull + 8ull * (lev - 1) + 16ull * __popc(bw_b);
+                b_ext += 4ull * bw_degree_sum(g, t, lev, e, bw_b) + 4ull * c;
+                b_out += 8ull * c;
+                b_need += 8ull * gr.W + 8ull;
+            }
+        }
+        cnt[e] = c;
+    }
+    if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
+}
+
+// level b+1 written from the rows: entry e's children G[A_e] at its exact offset
+// (ascending, the ordered layout every level of the trie keeps)
+__global__ void k_dlr_write(Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0, uint64_t e1,
+                            uint2* __restrict__ out) {
+    const uint64_t c0 = cpos_b[e0];
+    for (uint64_t e = e0 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e1; e += (uint64_t)gridDim.x * blockDim.x) {
+        const DlrGrp gr = dlr_group(a, e);
+        if (gr.m > (uint32_t)kDlrMaxM) continue;
+        const unsigned long long* r = a.R + gr.rb + (e - gr.g0) * gr.W;
+        uint64_t o = cpos_b[e] - c0;
+        for (uint32_t w = 0; w < gr.W; ++w) {
+            for (unsigned long long x = r[w]; x; x &= x - 1) {
+                const uint32_t s = 64u * w + (uint32_t)(__ffsll((long long)x) - 1);
+                out[o++] = make_uint2(a.lv[gr.g0 + s].x, (uint32_t)e);
+            }
+        }
+    }
+}
+
+// index of the rank-th set bit (0-based) of a W-word row
+__device__ __forceinline__ uint32_t dlr_select(const unsigned long long* r, uint32_t W, uint32_t rank) {
+    for (uint32_t w = 0; w < W; ++w) {
+        const unsigned long long x = r[w];
+        const uint32_t pc = (uint32_t)__popcll(x);
+        if (rank < pc) {
+            const uint32_t lo = (uint32_t)x, plo = (uint32_t)__popc(lo);
+            if (rank < plo) return 64u * w + (uint32_t)__fns(lo, 0, (int)rank + 1);
+            return 64u * w + 32u + (uint32_t)__fns((uint32_t)(x >> 32), 0, (int)(rank - plo) + 1);
+        }
+        rank -= pc;
+    }
+    return 0xffffffffu;
+}
+
+// level-(b+1) entry (e_t, G[s]): x = A_t & A_s; |L_{b+2}| += |x|; count += sum_{l in x} |x & A_l|
+// (WM: x held in registers for rows of up to WM words; WM = 0: re-read from the rows)
+template <int WM>
+__device__ __forceinline__ void dlr_tail_one(const unsigned long long* __restrict__ Rt,
+                                             const unsigned long long* __restrict__ Rs,
+                                             const unsigned long long* __restrict__ Rg, uint32_t W,
+                                             unsigned long long& lvl, unsigned long long& cnt) {
+    if constexpr (WM > 0) {
+        unsigned long long x[WM];
+#pragma unroll
+        for (int w = 0; w < WM; ++w) x[w] = (uint32_t)w < W ? (Rt[w] & Rs[w]) : 0ull;
+#pragma unroll
+        for (int w = 0; w < WM; ++w) {
+            lvl += __popcll(x[w]);
+            for (unsigned long long y = x[w]; y; y &= y - 1) {
+                const unsigned long long* Rl = Rg + (uint64_t)(64u * w + (uint32_t)(__ffsll((long long)y) - 1)) * W;
+                unsigned long long c = 0;
+#pragma unroll
+                for (int v = 0; v < WM; ++v) c += (uint32_t)v < W ? __popcll(x[v] & Rl[v]) : 0ull;
+                cnt += c;
+            }
+        }
+    } else {
+        for (uint32_t w = 0; w < W; ++w) {
+            const unsigned long long xw = Rt[w] & Rs[w];
+            lvl += __popcll(xw);
+            for (unsigned long long y = xw; y; y &= y - 1) {
+                const unsigned long long* Rl = Rg + (uint64_t)(64u * w + (uint32_t)(__ffsll((long long)y) - 1)) * W;
+                unsigned long long c = 0;
+                for (uint32_t v = 0; v < W; ++v) c += __popcll(Rt[v] & Rs[v] & Rl[v]);
+                cnt += c;
+            }
+        }
+    }
+}
+
+// thread per entry of the written level-(b+1) chunk out[0, size) (children of level-b
+// entries [e0, ..)): the two fused levels from the rows.  With count_bytes the §8.d
+// model of both: every level-(b+1) entry's extension and every level-(b+2) child's
+// count-only extension (lists of bw over the path, survivors, children written).
+template <bool count_bytes>
+__global__ void k_dlr_tail(Graph g, Trie t, Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0,
+                           const uint2* __restrict__ out, uint64_t size, unsigned long long* __restrict__ ctrl,
+                           uint32_t lev1, uint32_t bw1, uint32_t bw2) {
+    unsigned long long lvl = 0, cnt = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
+    const uint64_t c0 = cpos_b[e0];
+    for (uint64_t f = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; f < size; f += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t e = out[f].y;
+        const DlrGrp gr = dlr_group(a, e);
+        const unsigned long long* Rg = a.R + gr.rb;
+        const unsigned long long* Rt = Rg + (e - gr.g0) * gr.W;
+        const uint32_t s = dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0)));
+        const unsigned long long* Rs = Rg + (uint64_t)s * gr.W;
+        const unsigned long long lvl0 = lvl, cnt0 = cnt;
+        if (gr.W == 1) dlr_tail_one<1>(Rt, Rs, Rg, 1, lvl, cnt);
+        else if (gr.W == 2) dlr_tail_one<2>(Rt, Rs, Rg, 2, lvl, cnt);
+        else if (gr.W <= 4) dlr_tail_one<4>(Rt, Rs, Rg, gr.W, lvl, cnt);
+        else if (gr.W <= 8) dlr_tail_one<8>(Rt, Rs, Rg, gr.W, lvl, cnt);
+        else dlr_tail_one<0>(Rt, Rs, Rg, gr.W, lvl, cnt);
+        if (count_bytes) {
+            // level b+1 entry f (stored: walk the trie) and its |x| level-(b+2) children G[l]
+            const unsigned long long nx = lvl - lvl0, sx = cnt - cnt0;
+            const unsigned long long d1 = bw_degree_sum(g, t, lev1, f, bw1);
+            const unsigned long long d2 = bw_degree_sum(g, t, lev1, f, bw2 & ((1u << lev1) - 1u));
+            b_plan += 8ull + 8ull * (lev1 - 1) + 16ull * __popc(bw1) + nx * (8ull + 8ull * lev1 + 16ull * __popc(bw2));
+            b_ext += 4ull * d1 + 4ull * nx + 4ull * nx * d2 + 4ull * sx;
+            b_out += 8ull * nx;
+            b_need += 8ull + 16ull * gr.W + 8ull * nx * gr.W;
+            if ((bw2 >> lev1) & 1u) {     // the newest vertex's list: deg(G[l]) per child
+                for (uint32_t w = 0; w < gr.W; ++w)
+                    for (unsigned long long y = Rt[w] & Rs[w]; y; y &= y - 1)
+                        b_ext += 4ull * __ldg(g.deg + a.lv[gr.g0 + 64u * w + (uint32_t)(__ffsll((long long)y) - 1)].x);
+            }
+        }
+    }
+    lvl = warp_sum(lvl);
+    cnt = warp_sum(cnt);
+    if ((threadIdx.x & 31) == 0) {
+        if (lvl) atomicAdd(ctrl + kLrLevel, lvl);
+        add_u128(ctrl + kCountLo, cnt);
+    }
+    if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
+}
+
+// CUTS_DEBUG_GROUPS: log2 histogram of the children counts cnt[0..W) (the sizes of
+// the next level's sibling groups): per bucket the groups, sum m, sum m^2
+__global__ void k_group_hist(const uint64_t* __restrict__ cnt, uint32_t W, unsigned long long* __restrict__ h) {
+    __shared__ unsigned long long s[48];
+    if (threadIdx.x < 48) s[threadIdx.x] = 0;
+    __syncthreads();
+    for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < W; e += gridDim.x * blockDim.x) {
+        const unsigned long long m = cnt[e];
+        const int b = m ? min(15, 64 - __clzll((long long)m)) : 0;
+        atomicAdd(&s[b * 3], 1ull);
+        atomicAdd(&s[b * 3 + 1], m);
+        atomicAdd(&s[b * 3 + 2], m * m);
+    }
+    __syncthreads();
+    if (threadIdx.x < 48 && s[threadIdx.x]) atomicAdd(h + threadIdx.x, s[threadIdx.x]);
 }
 
 // ------------------------------------------------ SV intersection (ablation)

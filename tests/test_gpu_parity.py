@@ -599,3 +599,64 @@ def test_local_rows_group_size_tiers(cuts):
             assert c.stats()["level_size"] == lv, (q.name, flags)
         c.set_debug()
     c.close()
+
+
+def test_deep_local_rows_clique_tiers(cuts):
+    """Deep local rows (rows of the level-(k-3) sibling groups carry levels k-2, k-1 and
+    the count) on clique unions whose level-(k-3) groups span every row width:
+    K6 on K200 ∪ K70 ∪ K9 (groups of 198 / 68 / 7 members: 4-, 2- and 1-word rows),
+    K7 on K70 ∪ K12, K8 on K40 ∪ K11, each plus an ER component (oracle).  In K_n the
+    level sizes are n!/(n-j)!.  Default, CUTS_DEBUG_NO_DLR and CUTS_DEBUG_NO_LR agree at
+    a large arena and at a 96 MiB one (level k-2 cut into many entry-aligned chunks);
+    CUTS_DEBUG_NO_LR only where the windowed pipeline's pair count stays small."""
+    from math import perm
+    er = er_graph(60, 260, 11)
+    cases = ((6, (200, 70, 9)), (7, (70, 12)), (8, (40, 11)))
+    for k, sizes in cases:
+        edges, base = [], 0
+        for n in sizes:
+            edges += [(base + u, base + v) for u in range(n) for v in range(u + 1, n)]
+            base += n
+        edges += [(base + int(a), base + int(b)) for a, b in er.edge_list()]
+        g = graph_from_edges(base + er.n, edges)
+        q = dense_family(k)[0]
+        qe, qlv = oracle.count(er, q, levels=True)
+        want = sum(perm(n, k) for n in sizes) + qe
+        lv = [0] + [sum(perm(n, j) for n in sizes) + qlv[j] for j in range(1, k + 1)]
+        for arena in (8 << 30, 96 << 20):
+            c = cuts(device=0, arena_bytes=arena)
+            c.load_csr(g)
+            _set(c, q)
+            # the windowed pipeline (no local rows at all) only where its pair count is small
+            slow = perm(max(sizes), k - 1) > 2e9
+            for flags in ({}, {"no_dlr": True}) + (() if slow else ({"no_lr": True},)):
+                c.set_debug(**flags)
+                assert c.count("hybrid") == want, (k, arena, flags)
+                st = c.stats()
+                assert st["level_size"] == lv, (k, arena, flags)
+                if not flags and arena > (1 << 30):
+                    assert (st["fused_levels"] >> (k - 1)) & 1, "deep local rows did not run"
+            c.set_debug()
+            c.close()
+
+
+def test_deep_local_rows_large_group_fallback(cuts):
+    """A level-(k-3) group above the deep-rows limit (1,024 members) goes through the
+    windowed pipeline while the rest use rows: two adjacent hubs over a circulant
+    C_1100(1, 2, 3) give the hub pair a 1,100-member group at level 3 of K6 / K6-K2.
+    Counts and level sizes == oracle, default and CUTS_DEBUG_NO_DLR."""
+    n = 1100
+    edges = [(0, 1)] + [(h, 2 + i) for h in (0, 1) for i in range(n)]
+    edges += [(2 + i, 2 + (i + d) % n) for i in range(n) for d in (1, 2, 3)]
+    g = graph_from_edges(2 + n, edges)
+    c = cuts(device=0, arena_bytes=1 << 30)
+    c.load_csr(g)
+    for q in dense_family(6)[:2]:
+        want, lv = oracle.count(g, q, levels=True)
+        _set(c, q)
+        for flags in ({}, {"no_dlr": True}):
+            c.set_debug(**flags)
+            assert c.count("hybrid") == want, (q.name, flags)
+            assert c.stats()["level_size"] == lv, (q.name, flags)
+        c.set_debug()
+    c.close()

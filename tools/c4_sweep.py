@@ -66,6 +66,8 @@ def main():
                    "chunks": st["chunks"], "windows": st["windows"], "launches": st["launches"],
                    "ms_extend": round(st["ms_extend"], 1), "ms_plan": round(st["ms_plan"], 1),
                    "peak_arena_bytes": st["peak_arena_bytes"], "debug": args.debug, "rep": rep}
+            if flags.get("groups"):
+                rec["group_hist"] = {j: v for j, v in ctx.group_hist().items()}
             print(json.dumps(rec), flush=True)
             if out:
                 out.write(json.dumps(rec) + "\n")
