@@ -967,7 +967,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
             uint2* out = (uint2*)(ctx->arena + off);
             int t0 = -1;
             if (timing) { t0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[t0], ctx->stream)); }
-            const unsigned gw = (unsigned)std::min<uint64_t>((eb - ea + 255) / 256, (uint64_t)ctx->num_sms * 16);
+            const unsigned gw = (unsigned)std::min<uint64_t>((eb - ea + 7) / 8, (uint64_t)ctx->num_sms * 16);   // warp per entry
             k_dlr_write<<<gw, 256, 0, ctx->stream>>>(a, cposb, ea, eb, out);
             CK(cudaGetLastError());
             r.t.lv[J + 1] = out;

@@ -1311,20 +1311,28 @@ __global__ void k_dlr_counts(Graph g, Trie t, Dlr a, uint64_t* __restrict__ cnt,
 }
 
 // level b+1 written from the rows: entry e's children G[A_e] at its exact offset
-// (ascending, the ordered layout every level of the trie keeps)
-__global__ void k_dlr_write(Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0, uint64_t e1,
-                            uint2* __restrict__ out) {
+// (ascending, the ordered layout every level of the trie keeps).  A warp per entry:
+// lane i of u32 row word w owns member 32w+i, a ballot ranks the set bits, so the
+// member reads and the children stores are both coalesced.
+__global__ void __launch_bounds__(256) k_dlr_write(Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0, uint64_t e1,
+                                                   uint2* __restrict__ out) {
     const uint64_t c0 = cpos_b[e0];
-    for (uint64_t e = e0 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e1; e += (uint64_t)gridDim.x * blockDim.x) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t e = e0 + (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); e < e1; e += nw) {
         const DlrGrp gr = dlr_group(a, e);
-        if (gr.m > (uint32_t)kDlrMaxM) continue;
-        const unsigned long long* r = a.R + gr.rb + (e - gr.g0) * gr.W;
+        if (gr.m > (uint32_t)kDlrMaxM) continue;                     // warp-uniform
+        const uint32_t* r = (const uint32_t*)(a.R + gr.rb + (e - gr.g0) * gr.W);
         uint64_t o = cpos_b[e] - c0;
-        for (uint32_t w = 0; w < gr.W; ++w) {
-            for (unsigned long long x = r[w]; x; x &= x - 1) {
-                const uint32_t s = 64u * w + (uint32_t)(__ffsll((long long)x) - 1);
-                out[o++] = make_uint2(a.lv[gr.g0 + s].x, (uint32_t)e);
+        const uint32_t nw32 = (gr.m + 31) / 32;
+        for (uint32_t w = 0; w < nw32; ++w) {
+            const uint32_t x = r[w];
+            if (!x) continue;
+            if ((x >> lane) & 1u) {
+                const uint32_t rank = __popc(x & ((1u << lane) - 1u));
+                out[o + rank] = make_uint2(a.lv[gr.g0 + 32u * w + lane].x, (uint32_t)e);
             }
+            o += __popc(x);
         }
     }
 }
@@ -1344,37 +1352,53 @@ __device__ __forceinline__ uint32_t dlr_select(const unsigned long long* r, uint
     return 0xffffffffu;
 }
 
-// level-(b+1) entry (e_t, G[s]): x = A_t & A_s; |L_{b+2}| += |x|; count += sum_{l in x} |x & A_l|
-// (WM: x held in registers for rows of up to WM words; WM = 0: re-read from the rows)
+// bits strictly above position p in word w of a row
+__device__ __forceinline__ unsigned long long dlr_above(uint32_t p, uint32_t w) {
+    const uint32_t pw = p >> 6;
+    if (w < pw) return 0ull;
+    if (w > pw) return ~0ull;
+    return (p & 63u) == 63u ? 0ull : (~0ull << ((p & 63u) + 1u));
+}
+
+// The tail counts by symmetry.  The four positions b-1 .. b+2 = k-1 are pairwise adjacent
+// in Q with the same backward set outside (the Reuse::sym conditions), so the
+// completions of a group are exactly the ordered 4-cliques (G[t], G[s], G[l], G[u]) of
+// its adjacency: |L_{b+2}| gets 6 x (triangles t < s < l) and the count 24 x (4-cliques
+// t < s < l < u).  The level-(b+1) entry (e_t, G[s]) with t < s holds the ones whose
+// two smallest members are t, s: x = A_t & A_s & {> s}, triangles += |x|,
+// 4-cliques += sum_{l in x} |x & A_l & {> l}|; an entry with t > s holds none.
+// WM: x held in registers for rows of up to WM words (0: re-read from the rows).
 template <int WM>
 __device__ __forceinline__ void dlr_tail_one(const unsigned long long* __restrict__ Rt,
                                              const unsigned long long* __restrict__ Rs,
-                                             const unsigned long long* __restrict__ Rg, uint32_t W,
-                                             unsigned long long& lvl, unsigned long long& cnt) {
+                                             const unsigned long long* __restrict__ Rg, uint32_t W, uint32_t s,
+                                             unsigned long long& tri, unsigned long long& k4) {
     if constexpr (WM > 0) {
         unsigned long long x[WM];
 #pragma unroll
-        for (int w = 0; w < WM; ++w) x[w] = (uint32_t)w < W ? (Rt[w] & Rs[w]) : 0ull;
+        for (int w = 0; w < WM; ++w) x[w] = (uint32_t)w < W ? (Rt[w] & Rs[w] & dlr_above(s, (uint32_t)w)) : 0ull;
 #pragma unroll
         for (int w = 0; w < WM; ++w) {
-            lvl += __popcll(x[w]);
+            tri += __popcll(x[w]);
             for (unsigned long long y = x[w]; y; y &= y - 1) {
-                const unsigned long long* Rl = Rg + (uint64_t)(64u * w + (uint32_t)(__ffsll((long long)y) - 1)) * W;
-                unsigned long long c = 0;
+                const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                const unsigned long long* Rl = Rg + (uint64_t)l * W;
+                unsigned long long c = __popcll(x[w] & Rl[w] & dlr_above(l, (uint32_t)w));
 #pragma unroll
-                for (int v = 0; v < WM; ++v) c += (uint32_t)v < W ? __popcll(x[v] & Rl[v]) : 0ull;
-                cnt += c;
+                for (int v = w + 1; v < WM; ++v) c += (uint32_t)v < W ? __popcll(x[v] & Rl[v]) : 0ull;
+                k4 += c;
             }
         }
     } else {
-        for (uint32_t w = 0; w < W; ++w) {
-            const unsigned long long xw = Rt[w] & Rs[w];
-            lvl += __popcll(xw);
+        for (uint32_t w = s >> 6; w < W; ++w) {
+            const unsigned long long xw = Rt[w] & Rs[w] & dlr_above(s, w);
+            tri += __popcll(xw);
             for (unsigned long long y = xw; y; y &= y - 1) {
-                const unsigned long long* Rl = Rg + (uint64_t)(64u * w + (uint32_t)(__ffsll((long long)y) - 1)) * W;
-                unsigned long long c = 0;
-                for (uint32_t v = 0; v < W; ++v) c += __popcll(Rt[v] & Rs[v] & Rl[v]);
-                cnt += c;
+                const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                const unsigned long long* Rl = Rg + (uint64_t)l * W;
+                unsigned long long c = __popcll(xw & Rl[w] & dlr_above(l, w));
+                for (uint32_t v = w + 1; v < W; ++v) c += __popcll(Rt[v] & Rs[v] & Rl[v]);
+                k4 += c;
             }
         }
     }
@@ -1382,48 +1406,56 @@ __device__ __forceinline__ void dlr_tail_one(const unsigned long long* __restric
 
 // thread per entry of the written level-(b+1) chunk out[0, size) (children of level-b
 // entries [e0, ..)): the two fused levels from the rows.  With count_bytes the §8.d
-// model of both: every level-(b+1) entry's extension and every level-(b+2) child's
-// count-only extension (lists of bw over the path, survivors, children written).
+// model of both — computed per entry as the unshared pipeline would extend it: every
+// level-(b+1) entry's extension and every level-(b+2) child's count-only extension
+// (lists of bw over the path, survivors, children written).
 template <bool count_bytes>
 __global__ void k_dlr_tail(Graph g, Trie t, Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0,
                            const uint2* __restrict__ out, uint64_t size, unsigned long long* __restrict__ ctrl,
                            uint32_t lev1, uint32_t bw1, uint32_t bw2) {
-    unsigned long long lvl = 0, cnt = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
+    unsigned long long tri = 0, k4 = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
     const uint64_t c0 = cpos_b[e0];
     for (uint64_t f = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; f < size; f += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t e = out[f].y;
         const DlrGrp gr = dlr_group(a, e);
         const unsigned long long* Rg = a.R + gr.rb;
-        const unsigned long long* Rt = Rg + (e - gr.g0) * gr.W;
+        const uint32_t te = (uint32_t)(e - gr.g0);
+        const unsigned long long* Rt = Rg + (uint64_t)te * gr.W;
         const uint32_t s = dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0)));
         const unsigned long long* Rs = Rg + (uint64_t)s * gr.W;
-        const unsigned long long lvl0 = lvl, cnt0 = cnt;
-        if (gr.W == 1) dlr_tail_one<1>(Rt, Rs, Rg, 1, lvl, cnt);
-        else if (gr.W == 2) dlr_tail_one<2>(Rt, Rs, Rg, 2, lvl, cnt);
-        else if (gr.W <= 4) dlr_tail_one<4>(Rt, Rs, Rg, gr.W, lvl, cnt);
-        else if (gr.W <= 8) dlr_tail_one<8>(Rt, Rs, Rg, gr.W, lvl, cnt);
-        else dlr_tail_one<0>(Rt, Rs, Rg, gr.W, lvl, cnt);
+        if (te < s) {
+            if (gr.W == 1) dlr_tail_one<1>(Rt, Rs, Rg, 1, s, tri, k4);
+            else if (gr.W == 2) dlr_tail_one<2>(Rt, Rs, Rg, 2, s, tri, k4);
+            else if (gr.W <= 4) dlr_tail_one<4>(Rt, Rs, Rg, gr.W, s, tri, k4);
+            else dlr_tail_one<0>(Rt, Rs, Rg, gr.W, s, tri, k4);
+        }
         if (count_bytes) {
-            // level b+1 entry f (stored: walk the trie) and its |x| level-(b+2) children G[l]
-            const unsigned long long nx = lvl - lvl0, sx = cnt - cnt0;
+            // the unshared model: entry f extends to |A_t & A_s| children, each of which
+            // counts |A_t & A_s & A_l| (same §8.d terms as the pipeline would charge)
+            unsigned long long nx = 0, sx = 0, dl = 0;
+            for (uint32_t w = 0; w < gr.W; ++w) {
+                const unsigned long long xw = Rt[w] & Rs[w];
+                nx += __popcll(xw);
+                for (unsigned long long y = xw; y; y &= y - 1) {
+                    const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                    const unsigned long long* Rl = Rg + (uint64_t)l * gr.W;
+                    for (uint32_t v = 0; v < gr.W; ++v) sx += __popcll(Rt[v] & Rs[v] & Rl[v]);
+                    if ((bw2 >> lev1) & 1u) dl += __ldg(g.deg + a.lv[gr.g0 + l].x);
+                }
+            }
             const unsigned long long d1 = bw_degree_sum(g, t, lev1, f, bw1);
             const unsigned long long d2 = bw_degree_sum(g, t, lev1, f, bw2 & ((1u << lev1) - 1u));
             b_plan += 8ull + 8ull * (lev1 - 1) + 16ull * __popc(bw1) + nx * (8ull + 8ull * lev1 + 16ull * __popc(bw2));
-            b_ext += 4ull * d1 + 4ull * nx + 4ull * nx * d2 + 4ull * sx;
+            b_ext += 4ull * d1 + 4ull * nx + 4ull * nx * d2 + 4ull * dl + 4ull * sx;
             b_out += 8ull * nx;
-            b_need += 8ull + 16ull * gr.W + 8ull * nx * gr.W;
-            if ((bw2 >> lev1) & 1u) {     // the newest vertex's list: deg(G[l]) per child
-                for (uint32_t w = 0; w < gr.W; ++w)
-                    for (unsigned long long y = Rt[w] & Rs[w]; y; y &= y - 1)
-                        b_ext += 4ull * __ldg(g.deg + a.lv[gr.g0 + 64u * w + (uint32_t)(__ffsll((long long)y) - 1)].x);
-            }
+            b_need += 8ull + 16ull * gr.W + (te < s ? 8ull * nx * gr.W / 3 : 0ull);
         }
     }
-    lvl = warp_sum(lvl);
-    cnt = warp_sum(cnt);
+    tri = warp_sum(tri) * 6ull;
+    k4 = warp_sum(k4) * 24ull;
     if ((threadIdx.x & 31) == 0) {
-        if (lvl) atomicAdd(ctrl + kLrLevel, lvl);
-        add_u128(ctrl + kCountLo, cnt);
+        if (tri) atomicAdd(ctrl + kLrLevel, tri);
+        add_u128(ctrl + kCountLo, k4);
     }
     if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
 }
