@@ -69,6 +69,17 @@ def _peaks():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
 
 
+def _alu_peak():
+    """Word-op ceiling of the tail (tools/micro/alu_peak.cu measured on a B200, profiles/),
+    else derived from unit counts: 148 SMs x 8 word-ops/clk (16 POPC/clk/SM, 2 per 64-bit
+    word) x 1.965 GHz."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "alu_peak_b200.json")))
+        return d["word_ops_per_s"] / 1e9, "measured on B200 (tools/micro/alu_peak.cu, profiles/alu_peak_b200.json)"
+    except Exception:
+        return 148 * 8 * 1.965, "derived: 148 SMs x 8 word-ops/clk x 1.965 GHz (DESIGN.md §5)"
+
+
 def _ncu_record(workload: str):
     """ncu --set full figures for the dominant kernel on this workload (profiles/), if captured."""
     path = os.path.join(ROOT, "profiles", f"ncu_{workload.lower()}_extend.json")
@@ -187,9 +198,12 @@ def run_ours(args):
             sts.append(c.stats())
         return n, sts
 
+    tail = [0.0, 0]              # this step's k_dlr_tail ms and launches
+
     def step(timing=False):
         """One pass over every (graph, query): (local count, launches, ms_extend, extend launches, level sizes)."""
         total, launches, ms_ext, n_ext, fused = 0, 0, 0.0, 0, 0
+        tail[0] = tail[1] = 0
         levels = [0] * 9
         ctx.set_debug(timing=timing)
         pass_id[0] += 1
@@ -202,6 +216,8 @@ def run_ours(args):
                 for st in sts:
                     launches += st["launches"]
                     ms_ext += st["ms_extend"]
+                    tail[0] += st["ms_tail"]
+                    tail[1] += st["tail_launches"]
                     n_ext += st["extend_launches"]
                     fused |= st["fused_levels"]
                     for j, v in enumerate(st["level_size"]):
@@ -220,6 +236,7 @@ def run_ours(args):
     sampler = ClockSampler(local)
     sampler.start()
     times, counts, launches, ms_ext, n_ext, levels = [], [], 0, 0.0, 0, ([], 0)
+    ms_tail, n_tail = 0.0, 0
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for _ in range(args.steps):
         flush.fill_(1)                      # evict L2 between timed steps
@@ -233,6 +250,8 @@ def run_ours(args):
         launches += la
         ms_ext += me
         n_ext += ne
+        ms_tail += tail[0]
+        n_tail += tail[1]
     clocks = sampler.stop()
     barrier()
     step_ms_local = sum(times) / len(times)
@@ -274,7 +293,7 @@ def run_ours(args):
         ctx.load_graph(rp, cl)
 
     # algorithmic bytes of the dominant kernel (k_extend), instrumented untimed pass
-    alg_ext = alg_need = 0
+    alg_ext = alg_need = tail_ops = 0
     if not args.no_bytes:
         ctx.set_debug(bytes_=True)
         for (rp, cl), (g, qs) in zip(dev_graphs, graphs):
@@ -284,24 +303,39 @@ def run_ours(args):
                 for st in count_q(ctx, q, f"b{pass_id[0]}q{qi}")[1]:
                     alg_ext += st["alg_bytes_extend"]
                     alg_need += st["alg_bytes_extend_needed"]
+                    tail_ops += st["tail_word_ops"]
         ctx.set_debug()
         alg_ext = D.allreduce_count(alg_ext, device=dev)
         alg_need = D.allreduce_count(alg_need, device=dev)
+        tail_ops = D.allreduce_count(tail_ops, device=dev)
     peak, peak_src = _peaks()
     per_step_ext_ms = D.allreduce_max(ms_ext / args.steps, device=dev)
     achieved = alg_ext / (per_step_ext_ms / 1e3) / 1e9 if per_step_ext_ms > 0 and alg_ext else None
     achieved_need = alg_need / (per_step_ext_ms / 1e3) / 1e9 if per_step_ext_ms > 0 and alg_need else None
     ncu, ncu_src = _ncu_record(wl.name)
-    roof = {"bound": "hbm", "kernel": "k_extend", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": (achieved / peak) if achieved else None,
-            "traffic": ncu.get("dram_bytes_per_launch") if ncu else None,
-            "model": "SURVEY §8.d, frozen: per entry 4·d per backward list (every list read once, P:1086) "
-                     "+ 4 per intersection survivor + children written; per step over all levels and chunks",
-            "peak_source": peak_src, "alg_bytes_per_step": alg_ext,
-            "needed_bytes_per_step": alg_need, "achieved_needed": achieved_need,
-            "frac_needed": (achieved_need / peak) if achieved_need else None,
-            "extend_ms_per_step": per_step_ext_ms, "extend_launches_per_step": n_ext // args.steps,
-            "extend_share_of_step": per_step_ext_ms / step_ms if step_ms else None}
+    model = {"bound": "hbm", "kernels": "every extend kernel (k_extend, k_pairs, k_lr_*, k_dlr_*)",
+             "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
+             "model": "SURVEY §8.d, frozen: per entry 4·d per backward list (every list read once, P:1086) "
+                      "+ 4 per intersection survivor + children written; per step over all levels and chunks",
+             "peak_source": peak_src, "alg_bytes_per_step": alg_ext, "needed_bytes_per_step": alg_need,
+             "achieved_needed": achieved_need, "frac_needed": (achieved_need / peak) if achieved_need else None,
+             "extend_ms_per_step": per_step_ext_ms, "extend_launches_per_step": n_ext // args.steps,
+             "extend_share_of_step": per_step_ext_ms / step_ms if step_ms else None}
+    tail_ms = D.allreduce_max(ms_tail / args.steps, device=dev)
+    if tail_ms > 0 and tail_ops:
+        # the dominant kernel is the deep-local-rows tail: integer bit algebra on L1-resident
+        # rows, so its roofline is the ALU rate of its unit
+        apk, apk_src = _alu_peak()
+        ach = tail_ops / (tail_ms / 1e3) / 1e9
+        roof = {"bound": "alu", "kernel": "k_dlr_tail", "achieved": ach, "peak": apk, "unit": "Gword-op/s",
+                "frac": ach / apk, "traffic": ncu.get("dram_bytes_per_launch") if ncu else None,
+                "per_unit": "one 64-bit AND + POPC + add of the symmetric 4-clique bit algebra "
+                            "(count from the instrumented pass, CUTS_DEBUG_BYTES)",
+                "word_ops_per_step": tail_ops, "kernel_ms_per_step": tail_ms,
+                "launches_per_step": n_tail // args.steps, "share_of_step": tail_ms / step_ms if step_ms else None,
+                "peak_source": apk_src, "hbm_model_8d": model}
+    else:
+        roof = dict(model, kernel="k_extend", traffic=ncu.get("dram_bytes_per_launch") if ncu else None)
     if ncu:
         roof["ncu"] = dict(ncu, source=ncu_src)
 

@@ -102,6 +102,11 @@ typedef struct {
     uint64_t fused_levels;             /* bit j: level j was (at least partly) never stored —
                                           the local-rows tail counts it from the level j-1
                                           sibling rows (level_size[j] stays exact)           */
+    double   ms_tail;                  /* CUTS_DEBUG_TIMING: CUDA-event ms of the deep-local-
+                                          rows tail kernel (k_dlr_tail) alone                */
+    uint64_t tail_launches;            /* launches timed in ms_tail                         */
+    uint64_t tail_word_ops;            /* CUTS_DEBUG_BYTES: 64-bit AND+POPC word operations
+                                          of the tail's bit algebra (its ALU roofline unit)  */
 } cuts_stats;
 
 /* debug / instrumentation flags for cuts_set_debug */

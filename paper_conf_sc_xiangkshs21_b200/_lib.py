@@ -52,7 +52,9 @@ class cuts_stats(ctypes.Structure):
                 ("alg_bytes_plan", ctypes.c_uint64), ("hubs", ctypes.c_uint64),
                 ("hub_threshold", ctypes.c_uint64), ("donations", ctypes.c_uint64),
                 ("donated_entries", ctypes.c_uint64), ("alg_bytes_extend_needed", ctypes.c_uint64),
-                ("free_identity", ctypes.c_uint64), ("fused_levels", ctypes.c_uint64)]
+                ("free_identity", ctypes.c_uint64), ("fused_levels", ctypes.c_uint64),
+                ("ms_tail", ctypes.c_double), ("tail_launches", ctypes.c_uint64),
+                ("tail_word_ops", ctypes.c_uint64)]
 
 
 _lib = None

@@ -328,7 +328,8 @@ class Cuts:
             "alg_bytes_plan": s.alg_bytes_plan, "hubs": s.hubs, "hub_threshold": s.hub_threshold,
             "donations": s.donations, "donated_entries": s.donated_entries,
             "alg_bytes_extend_needed": s.alg_bytes_extend_needed, "free_identity": s.free_identity,
-            "fused_levels": s.fused_levels,
+            "fused_levels": s.fused_levels, "ms_tail": s.ms_tail, "tail_launches": s.tail_launches,
+            "tail_word_ops": s.tail_word_ops,
         }
 
     def trie_decode(self, ca_levels, pa_levels) -> torch.Tensor:

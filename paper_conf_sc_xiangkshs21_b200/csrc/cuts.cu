@@ -85,7 +85,7 @@ struct cuts_ctx {
     int extend_occ_blocks = 0;
     std::vector<cudaEvent_t> ev_pool;
     size_t ev_used = 0;
-    std::vector<std::pair<int, int>> ev_ext, ev_plan;
+    std::vector<std::pair<int, int>> ev_ext, ev_plan, ev_tail;
     // flat-prefix seeding (cuts_set_prefixes): run from level pre_j instead of level 1
     uint32_t pre_j = 0;
     uint64_t pre_count = 0;
@@ -894,17 +894,18 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
     const uint64_t ng = o.eb - o.ea;
     const int cb = (ctx->debug & CUTS_DEBUG_BYTES) ? 1 : 0;
     const bool timing = (ctx->debug & CUTS_DEBUG_TIMING) != 0;
-    Dlr a{r.t.lv[J], N, o.cpos, o.w0, o.ea, o.eb, nullptr, nullptr};
+    Dlr a{r.t.lv[J], N, o.cpos, o.w0, o.ea, o.eb, nullptr, nullptr, nullptr};
     size_t cub_bytes = 0;
     const uint64_t nscan = std::max<uint64_t>(ng, N) + 1;
     CK(cub::DeviceScan::ExclusiveSum(nullptr, cub_bytes, (uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)nscan, ctx->stream));
     uint64_t off;
-    TRY(alloc_top(ctx, align_up((ng + 1) * 8) * 2 + align_up((N + 1) * 8) * 2 + align_up(cub_bytes), &off));
+    TRY(alloc_top(ctx, align_up((ng + 1) * 8) * 2 + align_up((N + 1) * 8) * 3 + align_up(cub_bytes), &off));
     char* p = ctx->arena + off;
     uint64_t* rw = (uint64_t*)p; p += align_up((ng + 1) * 8);
     uint64_t* roff = (uint64_t*)p; p += align_up((ng + 1) * 8);
     uint64_t* cnt = (uint64_t*)p; p += align_up((N + 1) * 8);
     uint64_t* cposb = (uint64_t*)p; p += align_up((N + 1) * 8);
+    a.desc = (unsigned long long*)p; p += align_up((N + 1) * 8);
     void* cub_tmp = p;
     int e0 = -1;
     if (timing) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
@@ -925,6 +926,8 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
     a.R = (unsigned long long*)(ctx->arena + off);
     a.roff = roff;
     CK(cudaMemsetAsync(a.R, 0, words * 8, ctx->stream));
+    k_dlr_desc<<<(unsigned)std::min<uint64_t>((N + 255) / 256, (uint64_t)ctx->num_sms * 16), 256, 0, ctx->stream>>>(a);
+    CK(cudaGetLastError());
     const double avg = (double)N / (double)std::max<uint64_t>(ng, 1) / 2;     // members tested per entry
     auto go = [&](auto kern, int G) {
         static int occ[4] = {0, 0, 0, 0};
@@ -971,6 +974,8 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
             k_dlr_write<<<gw, 256, 0, ctx->stream>>>(a, cposb, ea, eb, out);
             CK(cudaGetLastError());
             r.t.lv[J + 1] = out;
+            int tm = -1;
+            if (timing) { tm = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[tm], ctx->stream)); }
             const unsigned gt = (unsigned)std::min<uint64_t>((size + 255) / 256, (uint64_t)ctx->num_sms * 16);
             if (cb) k_dlr_tail<true><<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
                                                                 (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
@@ -981,6 +986,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
                 const int t1 = next_event(ctx);
                 CK(cudaEventRecord(ctx->ev_pool[t1], ctx->stream));
                 ctx->ev_ext.push_back({t0, t1});
+                ctx->ev_tail.push_back({tm, t1});
             }
             ctx->st.level_size[J + 1] += size;
             ctx->st.chunks++;
@@ -1033,7 +1039,7 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
     if (last && sym_last(ctx, r, J)) return pairs_level(ctx, r, J, N);
     uint32_t skip_small = 0;
     bool dlr = false;
-    if (dlr_level(ctx, r, J) && free_bytes(ctx) >= N * 32 + (64ull << 20)) {   // the two scans + room
+    if (dlr_level(ctx, r, J) && free_bytes(ctx) >= N * 40 + (64ull << 20)) {   // scans + descriptors + room
         uint64_t large = 0;
         TRY(dlr_chunk(ctx, r, J, N, &large, &dlr));
         ctx->top = top_save;
@@ -1328,6 +1334,7 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     for (uint32_t i = 0; i < ctx->q.k; ++i) ctx->st.order[i] = ctx->q.S[i];
     ctx->ev_used = 0;
     ctx->ev_ext.clear();
+    ctx->ev_tail.clear();
     ctx->ev_plan.clear();
     if (!ctx->pre_j) TRY(ensure_canonical(ctx));
     ctx->bot = ctx->canon_valid ? ctx->run_off : ctx->base_off;
@@ -1432,7 +1439,16 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
             ms += f;
         }
         ctx->st.ms_plan = ms;
+        ms = 0;
+        for (auto& pr : ctx->ev_tail) {
+            float f = 0;
+            CK(cudaEventElapsedTime(&f, ctx->ev_pool[pr.first], ctx->ev_pool[pr.second]));
+            ms += f;
+        }
+        ctx->st.ms_tail = ms;
+        ctx->st.tail_launches = ctx->ev_tail.size();
     }
+    ctx->st.tail_word_ops = ctx->h_ctrl[kTailOps];
     ctx->st.ms_total = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
     return CUTS_OK;
 }

@@ -119,7 +119,7 @@ enum Mode { kWrite = 0, kCount = 1, kEnum = 2 };
 // ancestor range, or the set-difference searches), reported beside the model
 enum Ctrl { kCursor = 0, kCountLo = 1, kCountHi = 2, kErr = 3, kBytesPlan = 4, kBytesExt = 5,
             kEnumCursor = 6, kNumSel = 7, kWork = 8, kBytesOut = 9, kBytesNeed = 10, kFind = 24,
-            kBins = 12, kLrLevel = 15, kLrLarge = 29, kLrWork = 30, kDlrLarge = 31, kDlrWork = 32, kDistLimbs = 56, kCtrlWords = 64,
+            kBins = 12, kLrLevel = 15, kLrLarge = 29, kLrWork = 30, kDlrLarge = 31, kDlrWork = 32, kTailOps = 33, kDistLimbs = 56, kCtrlWords = 64,
             kGroupHist = 64, kGroupHistWords = 432 };   // CUTS_DEBUG_GROUPS: [level][16 buckets][3]
 
 __device__ __forceinline__ void add_u128(unsigned long long* lo_hi, unsigned long long v) {
@@ -1160,6 +1160,7 @@ struct Dlr {
     uint64_t w0, ea, eb;        // window start; parent slots [ea, eb) own the chunk (window-relative)
     const uint64_t* roff;       // row word offset of each parent slot's group (slot - ea)
     unsigned long long* R;      // rows
+    unsigned long long* desc;   // per entry: rb | te << 40 | m << 51 (k_dlr_desc); ~0: group too large
 };
 
 struct DlrGrp {
@@ -1169,14 +1170,27 @@ struct DlrGrp {
 };
 
 __device__ __forceinline__ DlrGrp dlr_group(const Dlr& a, uint64_t e) {
-    const uint64_t q = (uint64_t)a.lv[e].y - a.w0;
-    const uint64_t c0 = a.cpos[q], c1 = a.cpos[q + 1];
+    const unsigned long long d = a.desc[e];
     DlrGrp gr;
-    gr.g0 = c0 - a.cpos[a.ea];
-    gr.m = (uint32_t)(c1 - c0);
+    if (d == ~0ull) { gr.g0 = e; gr.rb = 0; gr.m = kDlrMaxM + 1; gr.W = 0; return gr; }
+    const uint32_t te = (uint32_t)(d >> 40) & 0x7ffu;
+    gr.g0 = e - te;
+    gr.rb = d & ((1ull << 40) - 1);
+    gr.m = (uint32_t)(d >> 51) & 0x7ffu;
     gr.W = (gr.m + 63) / 64;
-    gr.rb = a.roff[q - a.ea];
     return gr;
+}
+
+// per entry of the level-b chunk: its group's row base, its index in the group and the
+// group size, packed (one 8-byte load per entry for every later kernel)
+__global__ void k_dlr_desc(Dlr a) {
+    const uint64_t c0 = a.cpos[a.ea];
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t q = (uint64_t)a.lv[e].y - a.w0;
+        const uint64_t q0 = a.cpos[q], m = a.cpos[q + 1] - q0;
+        a.desc[e] = m > (uint64_t)kDlrMaxM ? ~0ull
+                                           : (a.roff[q - a.ea] | ((e - (q0 - c0)) << 40) | (m << 51));
+    }
 }
 
 // per parent slot: row words of its group (0 when it is left to the windowed pipeline)
@@ -1366,7 +1380,7 @@ __device__ __forceinline__ unsigned long long dlr_above(uint32_t p, uint32_t w) 
 // its adjacency: |L_{b+2}| gets 6 x (triangles t < s < l) and the count 24 x (4-cliques
 // t < s < l < u).  The level-(b+1) entry (e_t, G[s]) with t < s holds the ones whose
 // two smallest members are t, s: x = A_t & A_s & {> s}, triangles += |x|,
-// 4-cliques += sum_{l in x} |x & A_l & {> l}|; an entry with t > s holds none.
+// 4-cliques += sum_{l in x} |x & {> l} & A_l|; an entry with t > s holds none.
 // WM: x held in registers for rows of up to WM words (0: re-read from the rows).
 template <int WM>
 __device__ __forceinline__ void dlr_tail_one(const unsigned long long* __restrict__ Rt,
@@ -1380,10 +1394,11 @@ __device__ __forceinline__ void dlr_tail_one(const unsigned long long* __restric
 #pragma unroll
         for (int w = 0; w < WM; ++w) {
             tri += __popcll(x[w]);
-            for (unsigned long long y = x[w]; y; y &= y - 1) {
+            for (unsigned long long y = x[w]; y;) {
                 const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                y &= y - 1;                                   // the members of x above l in word w
                 const unsigned long long* Rl = Rg + (uint64_t)l * W;
-                unsigned long long c = __popcll(x[w] & Rl[w] & dlr_above(l, (uint32_t)w));
+                unsigned long long c = __popcll(y & Rl[w]);
 #pragma unroll
                 for (int v = w + 1; v < WM; ++v) c += (uint32_t)v < W ? __popcll(x[v] & Rl[v]) : 0ull;
                 k4 += c;
@@ -1393,10 +1408,11 @@ __device__ __forceinline__ void dlr_tail_one(const unsigned long long* __restric
         for (uint32_t w = s >> 6; w < W; ++w) {
             const unsigned long long xw = Rt[w] & Rs[w] & dlr_above(s, w);
             tri += __popcll(xw);
-            for (unsigned long long y = xw; y; y &= y - 1) {
+            for (unsigned long long y = xw; y;) {
                 const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                y &= y - 1;
                 const unsigned long long* Rl = Rg + (uint64_t)l * W;
-                unsigned long long c = __popcll(xw & Rl[w] & dlr_above(l, w));
+                unsigned long long c = __popcll(y & Rl[w]);
                 for (uint32_t v = w + 1; v < W; ++v) c += __popcll(Rt[v] & Rs[v] & Rl[v]);
                 k4 += c;
             }
@@ -1404,60 +1420,107 @@ __device__ __forceinline__ void dlr_tail_one(const unsigned long long* __restric
     }
 }
 
-// thread per entry of the written level-(b+1) chunk out[0, size) (children of level-b
-// entries [e0, ..)): the two fused levels from the rows.  With count_bytes the §8.d
-// model of both — computed per entry as the unshared pipeline would extend it: every
-// level-(b+1) entry's extension and every level-(b+2) child's count-only extension
-// (lists of bw over the path, survivors, children written).
+__device__ __forceinline__ void dlr_tail_item(const unsigned long long* __restrict__ R, unsigned long long rb,
+                                              uint32_t pk, unsigned long long& tri, unsigned long long& k4) {
+    const uint32_t te = pk & 0x7ffu, s = (pk >> 11) & 0x7ffu, W = pk >> 22;
+    const unsigned long long* Rg = R + rb;
+    const unsigned long long* Rt = Rg + (uint64_t)te * W;
+    const unsigned long long* Rs = Rg + (uint64_t)s * W;
+    if (W == 1) dlr_tail_one<1>(Rt, Rs, Rg, 1, s, tri, k4);
+    else if (W == 2) dlr_tail_one<2>(Rt, Rs, Rg, 2, s, tri, k4);
+    else if (W <= 4) dlr_tail_one<4>(Rt, Rs, Rg, W, s, tri, k4);
+    else dlr_tail_one<0>(Rt, Rs, Rg, W, s, tri, k4);
+}
+
+// Warps walk the written level-(b+1) chunk out[0, size) (children of level-b entries
+// [e0, ..)) 32 entries at a time; each lane resolves its entry (e_t, G[s]) — parent
+// from the trie, s = the rank-th member of A_t — and the entries with t < s go to a
+// warp-private queue in shared memory, which is drained 32 at a time, so every lane of
+// the bit-algebra loop holds work.  With count_bytes the §8.d model of both fused
+// levels, computed per entry as the unshared pipeline would charge it (every
+// level-(b+1) entry's extension and every level-(b+2) child's count-only extension).
 template <bool count_bytes>
-__global__ void k_dlr_tail(Graph g, Trie t, Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0,
-                           const uint2* __restrict__ out, uint64_t size, unsigned long long* __restrict__ ctrl,
-                           uint32_t lev1, uint32_t bw1, uint32_t bw2) {
-    unsigned long long tri = 0, k4 = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0;
+__global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0,
+                                                  const uint2* __restrict__ out, uint64_t size,
+                                                  unsigned long long* __restrict__ ctrl,
+                                                  uint32_t lev1, uint32_t bw1, uint32_t bw2) {
+    __shared__ unsigned long long q_rb[8][64];
+    __shared__ uint32_t q_pk[8][64];
+    unsigned long long tri = 0, k4 = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0, b_ops = 0;
     const uint64_t c0 = cpos_b[e0];
-    for (uint64_t f = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; f < size; f += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t e = out[f].y;
-        const DlrGrp gr = dlr_group(a, e);
-        const unsigned long long* Rg = a.R + gr.rb;
-        const uint32_t te = (uint32_t)(e - gr.g0);
-        const unsigned long long* Rt = Rg + (uint64_t)te * gr.W;
-        const uint32_t s = dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0)));
-        const unsigned long long* Rs = Rg + (uint64_t)s * gr.W;
-        if (te < s) {
-            if (gr.W == 1) dlr_tail_one<1>(Rt, Rs, Rg, 1, s, tri, k4);
-            else if (gr.W == 2) dlr_tail_one<2>(Rt, Rs, Rg, 2, s, tri, k4);
-            else if (gr.W <= 4) dlr_tail_one<4>(Rt, Rs, Rg, gr.W, s, tri, k4);
-            else dlr_tail_one<0>(Rt, Rs, Rg, gr.W, s, tri, k4);
-        }
-        if (count_bytes) {
-            // the unshared model: entry f extends to |A_t & A_s| children, each of which
-            // counts |A_t & A_s & A_l| (same §8.d terms as the pipeline would charge)
-            unsigned long long nx = 0, sx = 0, dl = 0;
-            for (uint32_t w = 0; w < gr.W; ++w) {
-                const unsigned long long xw = Rt[w] & Rs[w];
-                nx += __popcll(xw);
-                for (unsigned long long y = xw; y; y &= y - 1) {
-                    const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
-                    const unsigned long long* Rl = Rg + (uint64_t)l * gr.W;
-                    for (uint32_t v = 0; v < gr.W; ++v) sx += __popcll(Rt[v] & Rs[v] & Rl[v]);
-                    if ((bw2 >> lev1) & 1u) dl += __ldg(g.deg + a.lv[gr.g0 + l].x);
+    const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    uint32_t qn = 0;                                        // queued items (warp-uniform)
+    for (uint64_t base = (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; base < size; base += nwarps * 32) {
+        const uint64_t f = base + lane;
+        bool up = false;
+        unsigned long long rb = 0;
+        uint32_t pk = 0;
+        if (f < size) {
+            const uint32_t e = out[f].y;
+            const DlrGrp gr = dlr_group(a, e);
+            const uint32_t te = (uint32_t)(e - gr.g0);
+            const unsigned long long* Rt = a.R + gr.rb + (uint64_t)te * gr.W;
+            const uint32_t s = dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0)));
+            up = te < s;
+            rb = gr.rb;
+            pk = te | (s << 11) | (gr.W << 22);
+            if (count_bytes) {
+                // the unshared model: entry f extends to |A_t & A_s| children, each of which
+                // counts |A_t & A_s & A_l| (same §8.d terms as the pipeline would charge)
+                const unsigned long long* Rg = a.R + gr.rb;
+                const unsigned long long* Rs = Rg + (uint64_t)s * gr.W;
+                unsigned long long nx = 0, sx = 0, dl = 0;
+                for (uint32_t w = 0; w < gr.W; ++w) {
+                    const unsigned long long xw = Rt[w] & Rs[w];
+                    nx += __popcll(xw);
+                    for (unsigned long long y = xw; y; y &= y - 1) {
+                        const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                        const unsigned long long* Rl = Rg + (uint64_t)l * gr.W;
+                        for (uint32_t v = 0; v < gr.W; ++v) sx += __popcll(Rt[v] & Rs[v] & Rl[v]);
+                        if ((bw2 >> lev1) & 1u) dl += __ldg(g.deg + a.lv[gr.g0 + l].x);
+                    }
+                }
+                const unsigned long long d1 = bw_degree_sum(g, t, lev1, f, bw1);
+                const unsigned long long d2 = bw_degree_sum(g, t, lev1, f, bw2 & ((1u << lev1) - 1u));
+                b_plan += 8ull + 8ull * (lev1 - 1) + 16ull * __popc(bw1) + nx * (8ull + 8ull * lev1 + 16ull * __popc(bw2));
+                b_ext += 4ull * d1 + 4ull * nx + 4ull * nx * d2 + 4ull * dl + 4ull * sx;
+                b_out += 8ull * nx;
+                b_need += 8ull + 16ull * gr.W + (up ? 8ull * nx * gr.W / 3 : 0ull);
+                if (up) {     // word-ops of the symmetric bit algebra (the ALU roofline's unit)
+                    unsigned long long ops = gr.W - (s >> 6);
+                    for (uint32_t w = s >> 6; w < gr.W; ++w)
+                        for (unsigned long long y = Rt[w] & Rs[w] & dlr_above(s, w); y; y &= y - 1) ops += gr.W - w;
+                    b_ops += ops;
                 }
             }
-            const unsigned long long d1 = bw_degree_sum(g, t, lev1, f, bw1);
-            const unsigned long long d2 = bw_degree_sum(g, t, lev1, f, bw2 & ((1u << lev1) - 1u));
-            b_plan += 8ull + 8ull * (lev1 - 1) + 16ull * __popc(bw1) + nx * (8ull + 8ull * lev1 + 16ull * __popc(bw2));
-            b_ext += 4ull * d1 + 4ull * nx + 4ull * nx * d2 + 4ull * dl + 4ull * sx;
-            b_out += 8ull * nx;
-            b_need += 8ull + 16ull * gr.W + (te < s ? 8ull * nx * gr.W / 3 : 0ull);
+        }
+        const unsigned bal = __ballot_sync(0xffffffffu, up);
+        if (up) {
+            const uint32_t pos = qn + __popc(bal & ((1u << lane) - 1u));
+            q_rb[wq][pos] = rb;
+            q_pk[wq][pos] = pk;
+        }
+        qn += __popc(bal);
+        __syncwarp();
+        if (qn >= 32) {                                     // drain the 32 newest items
+            dlr_tail_item(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], tri, k4);
+            qn -= 32;
+            __syncwarp();
         }
     }
+    if ((uint32_t)lane < qn) dlr_tail_item(a.R, q_rb[wq][lane], q_pk[wq][lane], tri, k4);
     tri = warp_sum(tri) * 6ull;
     k4 = warp_sum(k4) * 24ull;
-    if ((threadIdx.x & 31) == 0) {
+    if (lane == 0) {
         if (tri) atomicAdd(ctrl + kLrLevel, tri);
         add_u128(ctrl + kCountLo, k4);
     }
-    if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
+    if (count_bytes) {
+        flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
+        b_ops = warp_sum(b_ops);
+        if (lane == 0 && b_ops) atomicAdd(ctrl + kTailOps, b_ops);
+    }
 }
 
 // CUTS_DEBUG_GROUPS: log2 histogram of the children counts cnt[0..W) (the sizes of
