@@ -144,6 +144,9 @@ typedef struct {
                                   clique-like count go through the ordered level-(k-3)
                                   extension and the (k-2)-level local rows instead of the
                                   level-(k-3) sibling rows carrying all three              */
+#define CUTS_DEBUG_TAIL_ALT 8192u /* ablation: the deep-local-rows tail gives one lane per
+                                  triangle (warp scan + shuffle search) instead of one lane
+                                  per level-(k-2) entry                                     */
 #define CUTS_DEBUG_GROUPS 2048u /* instrumentation: histogram of sibling-group sizes (children
                                   per entry) of every ordered level, read with
                                   cuts_debug_group_hist                                     */

@@ -970,17 +970,16 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
             uint2* out = (uint2*)(ctx->arena + off);
             int t0 = -1;
             if (timing) { t0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[t0], ctx->stream)); }
-            const unsigned gw = (unsigned)std::min<uint64_t>((eb - ea + 7) / 8, (uint64_t)ctx->num_sms * 16);   // warp per entry
+            const unsigned gw = (unsigned)std::min<uint64_t>((eb - ea + 15) / 16, (uint64_t)ctx->num_sms * 16);   // half-warp per entry
             k_dlr_write<<<gw, 256, 0, ctx->stream>>>(a, cposb, ea, eb, out);
             CK(cudaGetLastError());
             r.t.lv[J + 1] = out;
             int tm = -1;
             if (timing) { tm = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[tm], ctx->stream)); }
             const unsigned gt = (unsigned)std::min<uint64_t>((size + 255) / 256, (uint64_t)ctx->num_sms * 16);
-            if (cb) k_dlr_tail<true><<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
-                                                                (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
-            else k_dlr_tail<false><<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
-                                                                (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            auto kt = cb ? k_dlr_tail<true, 0> : ((ctx->debug & CUTS_DEBUG_TAIL_ALT) ? k_dlr_tail<false, 1> : k_dlr_tail<false, 0>);
+            kt<<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
+                                            (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
             CK(cudaGetLastError());
             if (timing) {
                 const int t1 = next_event(ctx);

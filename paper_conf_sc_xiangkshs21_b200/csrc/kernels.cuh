@@ -1325,26 +1325,30 @@ __global__ void k_dlr_counts(Graph g, Trie t, Dlr a, uint64_t* __restrict__ cnt,
 }
 
 // level b+1 written from the rows: entry e's children G[A_e] at its exact offset
-// (ascending, the ordered layout every level of the trie keeps).  A warp per entry:
-// lane i of u32 row word w owns member 32w+i, a ballot ranks the set bits, so the
-// member reads and the children stores are both coalesced.
+// (ascending, the ordered layout every level of the trie keeps).  A half-warp per entry
+// (two entries in flight per warp): lane i of the half owns member 16h+i of each 16-bit
+// slice h of the row, ranks come from a popcount of the slice below it, so the member
+// reads and the children stores are both coalesced.
 __global__ void __launch_bounds__(256) k_dlr_write(Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0, uint64_t e1,
                                                    uint2* __restrict__ out) {
-    const uint64_t c0 = cpos_b[e0];
-    const int lane = threadIdx.x & 31;
-    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t e = e0 + (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5); e < e1; e += nw) {
-        const DlrGrp gr = dlr_group(a, e);
-        if (gr.m > (uint32_t)kDlrMaxM) continue;                     // warp-uniform
-        const uint32_t* r = (const uint32_t*)(a.R + gr.rb + (e - gr.g0) * gr.W);
-        uint64_t o = cpos_b[e] - c0;
-        const uint32_t nw32 = (gr.m + 31) / 32;
-        for (uint32_t w = 0; w < nw32; ++w) {
-            const uint32_t x = r[w];
+    const uint64_t c0 = __ldg(cpos_b + e0);
+    const int lane = threadIdx.x & 31, hl = lane & 15;
+    const uint64_t nh = ((uint64_t)gridDim.x * blockDim.x) >> 4;
+    for (uint64_t e = e0 + (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 4); e < e1; e += nh) {
+        const unsigned long long d = __ldg(a.desc + e);
+        if (d == ~0ull) continue;                                    // half-warp-uniform
+        const uint32_t te = (uint32_t)(d >> 40) & 0x7ffu, m = (uint32_t)(d >> 51) & 0x7ffu;
+        const uint64_t g0 = e - te;
+        const uint32_t W = (m + 63) / 64;
+        const uint16_t* r = (const uint16_t*)(a.R + (d & ((1ull << 40) - 1)) + (uint64_t)te * W);
+        uint64_t o = __ldg(cpos_b + e) - c0;
+        const uint32_t nsl = (m + 15) / 16;
+        for (uint32_t h = 0; h < nsl; ++h) {
+            const uint32_t x = __ldg(r + h);
             if (!x) continue;
-            if ((x >> lane) & 1u) {
-                const uint32_t rank = __popc(x & ((1u << lane) - 1u));
-                out[o + rank] = make_uint2(a.lv[gr.g0 + 32u * w + lane].x, (uint32_t)e);
+            if ((x >> hl) & 1u) {
+                const uint32_t rank = __popc(x & ((1u << hl) - 1u));
+                out[o + rank] = make_uint2(__ldg(&a.lv[g0 + 16u * h + hl].x), (uint32_t)e);
             }
             o += __popc(x);
         }
@@ -1432,6 +1436,85 @@ __device__ __forceinline__ void dlr_tail_item(const unsigned long long* __restri
     else dlr_tail_one<0>(Rt, Rs, Rg, W, s, tri, k4);
 }
 
+// bit position of the rank-th (0-based) set bit of y (rank < popc(y))
+__device__ __forceinline__ uint32_t dlr_fns64(unsigned long long y, uint32_t rank) {
+    const uint32_t lo = (uint32_t)y, plo = (uint32_t)__popc(lo);
+    return rank < plo ? (uint32_t)__fns(lo, 0, (int)rank + 1) : 32u + (uint32_t)__fns((uint32_t)(y >> 32), 0, (int)(rank - plo) + 1);
+}
+
+// CUTS_DEBUG_TAIL_ALT (ablation): drain the 32 queued entries with one lane per
+// triangle instead of one lane per entry — each entry's x (rows of <= 4 words) is staged in
+// the warp's shared memory, a warp scan numbers the triangles, every round gives each lane
+// one (binary search of the scan by shuffles) and the lane adds |x & {> l} & A_l|.
+// Entries with wider rows keep the per-entry loop.
+__device__ __forceinline__ void dlr_drain_tri(const unsigned long long* __restrict__ R, unsigned long long rb, uint32_t pk,
+                                              bool own, unsigned long long* xs, unsigned long long& tri,
+                                              unsigned long long& k4) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t te = pk & 0x7ffu, s = (pk >> 11) & 0x7ffu, W = pk >> 22;
+    const unsigned long long* Rg = R + rb;
+    uint32_t n = 0;
+    if (own && W > 4) dlr_tail_item(R, rb, pk, tri, k4);
+    if (own && W <= 4) {
+        const unsigned long long* Rt = Rg + (uint64_t)te * W;
+        const unsigned long long* Rs = Rg + (uint64_t)s * W;
+#pragma unroll
+        for (int w = 0; w < 4; ++w) {
+            const unsigned long long xw = (uint32_t)w < W ? (Rt[w] & Rs[w] & dlr_above(s, (uint32_t)w)) : 0ull;
+            xs[lane * 4 + w] = xw;
+            n += (uint32_t)__popcll(xw);
+        }
+        tri += n;
+    }
+    uint32_t incl = n;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
+    }
+    const uint32_t excl = incl - n;
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    __syncwarp();
+    for (uint32_t j = 0; j < total; j += 32) {
+        const uint32_t k = j + lane;
+        uint32_t o = 0;
+#pragma unroll
+        for (uint32_t step = 16; step; step >>= 1) {
+            const uint32_t v = __shfl_sync(0xffffffffu, incl, (int)(o + step - 1));
+            if (v <= k) o += step;
+        }
+        uint32_t r = k - __shfl_sync(0xffffffffu, excl, (int)o);
+        const unsigned long long orb = __shfl_sync(0xffffffffu, rb, (int)o);
+        const uint32_t Wo = __shfl_sync(0xffffffffu, pk, (int)o) >> 22;
+        if (k < total) {
+            unsigned long long x[4];
+#pragma unroll
+            for (int w = 0; w < 4; ++w) x[w] = xs[o * 4 + w];
+            uint32_t wl = 0;
+#pragma unroll
+            for (int w = 0; w < 4; ++w) {                   // the word holding the r-th member
+                const uint32_t pc = (uint32_t)__popcll(x[w]);
+                if (wl == (uint32_t)w && r >= pc) { r -= pc; wl = w + 1; }
+            }
+            unsigned long long xl = 0;
+#pragma unroll
+            for (int w = 0; w < 4; ++w) xl = (uint32_t)w == wl ? x[w] : xl;
+            const uint32_t b = dlr_fns64(xl, r);
+            const uint32_t l = 64u * wl + b;
+            const unsigned long long* Rl = R + orb + (uint64_t)l * Wo;
+            unsigned long long c = 0;
+#pragma unroll
+            for (int w = 0; w < 4; ++w) {
+                const unsigned long long m = (uint32_t)w < wl ? 0ull
+                                           : ((uint32_t)w == wl ? (b == 63u ? 0ull : (~0ull << (b + 1u))) : ~0ull);
+                c += ((uint32_t)w < Wo && m) ? __popcll(x[w] & m & Rl[w]) : 0ull;
+            }
+            k4 += c;
+        }
+    }
+    __syncwarp();
+}
+
 // Warps walk the written level-(b+1) chunk out[0, size) (children of level-b entries
 // [e0, ..)) 32 entries at a time; each lane resolves its entry (e_t, G[s]) — parent
 // from the trie, s = the rank-th member of A_t — and the entries with t < s go to a
@@ -1439,13 +1522,14 @@ __device__ __forceinline__ void dlr_tail_item(const unsigned long long* __restri
 // the bit-algebra loop holds work.  With count_bytes the §8.d model of both fused
 // levels, computed per entry as the unshared pipeline would charge it (every
 // level-(b+1) entry's extension and every level-(b+2) child's count-only extension).
-template <bool count_bytes>
+template <bool count_bytes, int V>
 __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0,
                                                   const uint2* __restrict__ out, uint64_t size,
                                                   unsigned long long* __restrict__ ctrl,
                                                   uint32_t lev1, uint32_t bw1, uint32_t bw2) {
     __shared__ unsigned long long q_rb[8][64];
     __shared__ uint32_t q_pk[8][64];
+    __shared__ unsigned long long q_x[V ? 8 : 1][V ? 128 : 1];   // CUTS_DEBUG_TAIL_ALT: staged x words
     unsigned long long tri = 0, k4 = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0, b_ops = 0;
     const uint64_t c0 = cpos_b[e0];
     const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
@@ -1504,12 +1588,18 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
         qn += __popc(bal);
         __syncwarp();
         if (qn >= 32) {                                     // drain the 32 newest items
-            dlr_tail_item(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], tri, k4);
+            if (V) dlr_drain_tri(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], true, q_x[V ? wq : 0], tri, k4);
+            else dlr_tail_item(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], tri, k4);
             qn -= 32;
             __syncwarp();
         }
     }
-    if ((uint32_t)lane < qn) dlr_tail_item(a.R, q_rb[wq][lane], q_pk[wq][lane], tri, k4);
+    if (V) {
+        if (qn) dlr_drain_tri(a.R, (uint32_t)lane < qn ? q_rb[wq][lane] : 0ull, (uint32_t)lane < qn ? q_pk[wq][lane] : 0u,
+                              (uint32_t)lane < qn, q_x[V ? wq : 0], tri, k4);
+    } else if ((uint32_t)lane < qn) {
+        dlr_tail_item(a.R, q_rb[wq][lane], q_pk[wq][lane], tri, k4);
+    }
     tri = warp_sum(tri) * 6ull;
     k4 = warp_sum(k4) * 24ull;
     if (lane == 0) {

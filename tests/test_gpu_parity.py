@@ -608,6 +608,7 @@ def test_deep_local_rows_clique_tiers(cuts):
     K7 on K70 ∪ K12, K8 on K40 ∪ K11, each plus an ER component (oracle).  In K_n the
     level sizes are n!/(n-j)!.  Default, CUTS_DEBUG_NO_DLR and CUTS_DEBUG_NO_LR agree at
     a large arena and at a 96 MiB one (level k-2 cut into many entry-aligned chunks);
+    CUTS_DEBUG_TAIL_ALT (lane per triangle) likewise;
     CUTS_DEBUG_NO_LR only where the windowed pipeline's pair count stays small."""
     from math import perm
     er = er_graph(60, 260, 11)
@@ -629,7 +630,7 @@ def test_deep_local_rows_clique_tiers(cuts):
             _set(c, q)
             # the windowed pipeline (no local rows at all) only where its pair count is small
             slow = perm(max(sizes), k - 1) > 2e9
-            for flags in ({}, {"no_dlr": True}) + (() if slow else ({"no_lr": True},)):
+            for flags in ({}, {"tail_alt": True}, {"no_dlr": True}) + (() if slow else ({"no_lr": True},)):
                 c.set_debug(**flags)
                 assert c.count("hybrid") == want, (k, arena, flags)
                 st = c.stats()
