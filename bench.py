@@ -48,6 +48,9 @@ def _args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--chunks-per-rank", type=int, default=16, help="dynamic root queue granularity (N > 1)")
     ap.add_argument("--no-donate", action="store_true", help="N > 1: root queue only (no Alg. 3 donations)")
+    ap.add_argument("--partition-depth", type=int, default=3,
+                    help="N > 1: the dynamic queue hands out chunks of the shuffled level-D list "
+                         "(cuts_set_partition_depth; 1 = the paper's level-1 roots)")
     ap.add_argument("--e2e-steps", type=int, default=3, help="steps of the end-to-end (host buffers) leg")
     ap.add_argument("--cpu-budget", type=float, default=20.0, help="seconds of oracle work per cpu_baseline leg")
     ap.add_argument("--no-bytes", action="store_true", help="skip the instrumented algorithmic-bytes pass")
@@ -171,16 +174,18 @@ def run_ours(args):
     donations = [0, 0]          # donations made, prefix rows shipped (this rank)
 
     def count_q(c, q, tag):
-        """This rank's share of one query.  N = 1: the whole root range.  N > 1: root
-        chunks of the shuffled level-1 list pulled from a shared atomic counter, then
-        Alg. 3 donations to idle ranks (flat prefixes over gloo)."""
+        """This rank's share of one query.  N = 1: the whole root range.  N > 1: chunks of
+        the shuffled level-D list (D = --partition-depth; D = 1 is the paper's root
+        partition) pulled from a shared atomic counter, then Alg. 3 donations to idle
+        ranks (flat prefixes over gloo)."""
         qr, qc = q.csr()
         c.set_query(qr, qc)
         if wl.root_range is not None:                 # stated root range (C4)
             c.set_root_range(*wl.roots(c.level1_size()[0]))
         if world == 1:
             return c.count(wl.mode), [c.stats()]
-        _, l1 = c.level1_size()
+        c.set_partition_depth(args.partition_depth)
+        l1 = c.partition_size()                     # |L_D| over the root range
         cs = max(1, -(-l1 // (world * args.chunks_per_rank)))
         queue = D.RootQueue(store, tag, D.n_chunks(l1, cs))
         if donate:
@@ -351,7 +356,8 @@ def run_ours(args):
                    "deepest_stored_level_entries": deepest, "deepest_stored_level_bytes": 8 * deepest,
                    "bfs_trie_bytes_at_largest_level": 8 * max(levels[1:kmax], default=0),
                    "parallelism": (f"NCCL world {world} via cuts_set_dist; dynamic root-chunk queue "
-                                   f"({args.chunks_per_rank} chunks/rank/query)"
+                                   f"({args.chunks_per_rank} chunks/rank/query of the shuffled level-"
+                                   f"{args.partition_depth} list)"
                                    + (" + Alg. 3 prefix donations (store control plane, gloo host data plane)"
                                       if donate else "")
                                    + " + cuts_allreduce_count" if world > 1 else "1 GPU"),

@@ -252,6 +252,22 @@ cuts_status cuts_count(cuts_ctx* ctx, cuts_mode mode, uint64_t* out);
 cuts_status cuts_enumerate(cuts_ctx* ctx, cuts_mode mode, uint32_t* d_out,
                            uint64_t cap_rows, uint64_t* n_found);
 
+/* Multi-GPU partition below level 1 (an extension of the paper's first-level partition,
+ * P:1277-1279, for power-law roots whose subtrees differ by orders of magnitude): with
+ * depth D > 1 every count/enumerate builds levels 1..D whole over the root range (BFS,
+ * identical on every part), shuffles level D with the seeded bijection and
+ * applies the cuts_set_root_slice (begin, end, part, nparts) — or the cuts_set_dist
+ * default — to THAT list, then extends the slice (HYBRID or BFS) from flat prefixes.
+ * Summed over the parts of a partition the counts equal the unpartitioned count and the
+ * level sizes are exact (levels < D are reported by the part holding shuffled position 0
+ * only).  D = 1 (default) slices the level-1 list; D >= k behaves like 1.  CUTS_EINVAL
+ * unless 1 <= D < 8.  Persists across queries. */
+cuts_status cuts_set_partition_depth(cuts_ctx* ctx, uint32_t depth);
+
+/* Size of the list the slice partitions: |L_D| over the root range for the current
+ * query and partition depth (|L_1| in range for D = 1); runs the BFS to level D. */
+cuts_status cuts_partition_size(cuts_ctx* ctx, uint64_t* n);
+
 /* Stats of the last count/enumerate. */
 cuts_status cuts_get_stats(const cuts_ctx* ctx, cuts_stats* out);
 

@@ -28,7 +28,7 @@ EXPORTED = ["cuts_version", "cuts_create", "cuts_destroy", "cuts_last_error", "c
             "cuts_set_query", "cuts_set_root_range", "cuts_set_root_slice", "cuts_level1_size", "cuts_count",
             "cuts_enumerate", "cuts_get_stats", "cuts_set_debug", "cuts_trie_decode", "cuts_set_hub_threshold",
             "cuts_set_prefixes", "cuts_set_donation", "cuts_dist_unique_id", "cuts_set_dist",
-            "cuts_allreduce_count", "cuts_debug_group_hist"]
+            "cuts_allreduce_count", "cuts_debug_group_hist", "cuts_set_partition_depth", "cuts_partition_size"]
 
 # callback types of cuts_set_donation
 POLL_FN = ctypes.CFUNCTYPE(ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64)
@@ -94,6 +94,8 @@ def load() -> ctypes.CDLL:
         "cuts_set_dist": ([P, i32, i32, P, P], i32),
         "cuts_allreduce_count": ([P, u64, u64, u64p, u64p], i32),
         "cuts_debug_group_hist": ([P, u64p], i32),
+        "cuts_set_partition_depth": ([P, u32], i32),
+        "cuts_partition_size": ([P, u64p], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

@@ -260,6 +260,17 @@ class Cuts:
                                                   ctypes.byref(lo), ctypes.byref(hi)))
         return int(lo.value) | (int(hi.value) << 64)
 
+    def set_partition_depth(self, depth: int = 1):
+        """cuts_set_partition_depth: the root slice applies to the shuffled level-`depth` list."""
+        self._check(self.lib.cuts_set_partition_depth(self.h, int(depth)))
+        return self
+
+    def partition_size(self) -> int:
+        """|L_depth| over the root range (the list cuts_set_root_slice partitions)."""
+        n = ctypes.c_uint64()
+        self._check(self.lib.cuts_partition_size(self.h, ctypes.byref(n)))
+        return int(n.value)
+
     def level1_size(self):
         """(canonical level-1 size, size inside the root range) for the current query."""
         a, b = ctypes.c_uint64(), ctypes.c_uint64()

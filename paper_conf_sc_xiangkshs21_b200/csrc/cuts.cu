@@ -78,6 +78,8 @@ struct cuts_ctx {
     uint64_t root_begin = 0, root_end = ~0ull;
     uint64_t slice_begin = 0, slice_end = ~0ull;
     uint32_t part = 0, nparts = 1;
+    uint32_t part_depth = 1;               // level whose shuffled list the slice partitions
+    bool size_only = false;                // cuts_partition_size: stop after the partition level
     uint32_t debug = 0;
     // run state
     uint64_t bot = 0, top = 0, peak = 0;
@@ -1090,10 +1092,11 @@ cuts_status hybrid_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
 }
 
 // BFS: every level stored whole (Alg. 1); ENOMEM when a level does not fit
-cuts_status bfs_levels(cuts_ctx* ctx, Run& r, int J0, uint64_t N1) {
+cuts_status bfs_levels(cuts_ctx* ctx, Run& r, int J0, uint64_t N1, int jstop = 0) {
     const int k = (int)ctx->q.k;
     uint64_t N = N1;
-    for (int J = J0; J <= k - 1 && N > 0; ++J) {
+    const int jend = jstop ? jstop : k;           // extend J -> J+1 while J < jend
+    for (int J = J0; J < jend && J <= k - 1 && N > 0; ++J) {
         const bool last = (J == k - 1);
         const uint64_t top_save = ctx->top;
         uint64_t W = pick_window(ctx, N);
@@ -1108,11 +1111,35 @@ cuts_status bfs_levels(cuts_ctx* ctx, Run& r, int J0, uint64_t N1) {
             out = (uint2*)(ctx->arena + off);
             CK(cudaMemsetAsync(ctx->ctrl + kCursor, 0, sizeof(unsigned long long), ctx->stream));
         }
+        uint64_t run = 0;                   // jstop: entries written so far (ordered levels)
         for (uint64_t w0 = 0; w0 < N; w0 += W) {
             w.w0 = w0;
             w.W = (uint32_t)std::min<uint64_t>(W, N - w0);
             TRY(plan_window(ctx, r, J, w));
             if (last) TRY(extend_last(ctx, r, J, w, r.enumerate ? kEnum : kCount));
+            else if (jstop) {
+                // the partition prefix (cuts_set_partition_depth) must be the same list on
+                // every part: write it ORDERED (per-entry counts, scan, children at exact
+                // offsets in candidate order) instead of by warp-aggregated atomics
+                CK(cudaMemsetAsync(w.ub, 0, (w.W + 1) * sizeof(uint64_t), ctx->stream));
+                Window wa = w;
+                wa.ord_cnt = w.ub;
+                TRY(extend_range(ctx, r, J, wa, 0, w.total, kCount, nullptr, 0));
+                CK(cub::DeviceScan::ExclusiveSum(w.cub_tmp, w.cub_bytes, w.ub, w.cpos, (int64_t)w.W + 1, ctx->stream));
+                CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 1, w.cpos + w.W, 8, cudaMemcpyDeviceToHost, ctx->stream));
+                CK(cudaStreamSynchronize(ctx->stream));
+                const uint64_t sz = ctx->h_ctrl[kCtrlWords + 1];
+                if (run + sz > cap)
+                    return fail(ctx, CUTS_ENOMEM, "partition prefix: level %d does not fit the arena", J + 1);
+                Window wb = w;
+                wb.ord_pos = w.cpos;
+                wb.ord_ea = 0;
+                TRY(extend_range(ctx, r, J, wb, 0, w.total, kWrite, out + run, sz));
+                run += sz;
+                ctx->h_ctrl[kCursor] = run;
+                CK(cudaMemcpyAsync(ctx->ctrl + kCursor, ctx->h_ctrl + kCursor, 8, cudaMemcpyHostToDevice, ctx->stream));
+                continue;
+            }
             else TRY(extend_range(ctx, r, J, w, 0, w.total, kWrite, out, cap));
             if (!last && w0 + W < N) {     // stop at the first window that overflows the level
                 CK(cudaMemcpyAsync(ctx->h_ctrl + kCursor, ctx->ctrl + kCursor, 8, cudaMemcpyDeviceToHost, ctx->stream));
@@ -1217,6 +1244,37 @@ cuts_status ensure_canonical(cuts_ctx* ctx) {
 }
 
 // level 1: canonical list -> root range -> shuffle -> slice
+// seeded Feistel bijection of [0, R) (reading P25)
+Shuffle make_shuffle(uint64_t seed, uint64_t R) {
+    Shuffle sh{};
+    sh.R = R;
+    uint32_t bits = 2;
+    while ((1ull << bits) < R) ++bits;
+    if (bits & 1) ++bits;
+    sh.half = bits / 2;
+    sh.mask = (uint32_t)((1ull << sh.half) - 1);
+    uint64_t x = seed;
+    for (int i = 0; i < 4; ++i) {   // splitmix64 round keys
+        x += 0x9E3779B97F4A7C15ull;
+        uint64_t z = x;
+        z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+        z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+        sh.key[i] = z ^ (z >> 31);
+    }
+    return sh;
+}
+
+// positions [sb, se) of a list of R with p % nparts == part: first position, count
+void slice_of(const cuts_ctx* ctx, uint64_t R, uint64_t* p0, uint64_t* cnt) {
+    const uint64_t sb = std::min(ctx->slice_begin, R), se = std::min(ctx->slice_end, R);
+    *p0 = 0;
+    *cnt = 0;
+    if (se > sb) {
+        *p0 = sb + ((ctx->part + ctx->nparts - (uint32_t)(sb % ctx->nparts)) % ctx->nparts);
+        *cnt = *p0 < se ? (se - *p0 + ctx->nparts - 1) / ctx->nparts : 0;
+    }
+}
+
 cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
     const uint32_t* canon = ctx->canon;
     const uint64_t ncanon = ctx->canon_n;
@@ -1225,31 +1283,13 @@ cuts_status build_level1(cuts_ctx* ctx, Run& r, uint64_t* n1) {
     if (re < rb) re = rb;
     const uint64_t R = re - rb;
     // slice of shuffled positions [sb, se) with p % nparts == part
-    uint64_t sb = std::min(ctx->slice_begin, R), se = std::min(ctx->slice_end, R);
     uint64_t cnt = 0, p0 = 0;
-    if (se > sb) {
-        p0 = sb + ((ctx->part + ctx->nparts - (uint32_t)(sb % ctx->nparts)) % ctx->nparts);
-        cnt = p0 < se ? (se - p0 + ctx->nparts - 1) / ctx->nparts : 0;
-    }
+    slice_of(ctx, R, &p0, &cnt);
     uint64_t off_l1;
     TRY(alloc_bot(ctx, std::max<uint64_t>(cnt, 1) * sizeof(uint2), &off_l1));
     uint2* L1 = (uint2*)(ctx->arena + off_l1);
     if (cnt) {
-        Shuffle sh{};
-        sh.R = R;
-        uint32_t bits = 2;
-        while ((1ull << bits) < R) ++bits;
-        if (bits & 1) ++bits;
-        sh.half = bits / 2;
-        sh.mask = (uint32_t)((1ull << sh.half) - 1);
-        uint64_t x = ctx->seed;
-        for (int i = 0; i < 4; ++i) {   // splitmix64 round keys
-            x += 0x9E3779B97F4A7C15ull;
-            uint64_t z = x;
-            z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
-            z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
-            sh.key[i] = z ^ (z >> 31);
-        }
+        const Shuffle sh = make_shuffle(ctx->seed, R);
         unsigned grid = (unsigned)std::min<uint64_t>((cnt + 255) / 256, (uint64_t)ctx->num_sms * 8);
         k_level1<<<grid, 256, 0, ctx->stream>>>(canon, rb, sh, p0, ctx->nparts, cnt, L1);
         CK(cudaGetLastError());
@@ -1303,9 +1343,7 @@ cuts_status build_free_lists(cuts_ctx* ctx, Run& r) {
 }
 
 // flat-prefix seeding: levels 1..pre_j as a chain trie over the caller's rows
-cuts_status build_prefix_levels(cuts_ctx* ctx, Run& r) {
-    const uint32_t J = ctx->pre_j;
-    const uint64_t cnt = ctx->pre_count;
+cuts_status build_prefix_levels(cuts_ctx* ctx, Run& r, uint32_t J, uint64_t cnt, const uint32_t* rows) {
     for (uint32_t l = 1; l <= J; ++l) {
         uint64_t off;
         TRY(alloc_bot(ctx, std::max<uint64_t>(cnt, 1) * sizeof(uint2), &off));
@@ -1314,11 +1352,67 @@ cuts_status build_prefix_levels(cuts_ctx* ctx, Run& r) {
     }
     if (cnt) {
         unsigned grid = (unsigned)std::min<uint64_t>((cnt + 255) / 256, (uint64_t)ctx->num_sms * 8);
-        k_prefix_import<<<grid, 256, 0, ctx->stream>>>(ctx->pre_rows, J, cnt, r.t);
+        k_prefix_import<<<grid, 256, 0, ctx->stream>>>(rows, J, cnt, r.t);
         CK(cudaGetLastError());
         ctx->st.launches++;
     }
     return CUTS_OK;
+}
+
+// cuts_set_partition_depth D > 1: levels 1..D are built whole (BFS over the root range,
+// the same on every part), the seeded shuffle of level D is sliced like the level-1 list
+// (P:1277-1279 one level down) and the slice is extended from flat prefixes.  Levels
+// below D are reported only by the part holding shuffled position 0 (part 0 of the slice
+// that starts at 0), so summing the stats of all parts gives the exact level sizes.
+cuts_status partition_run(cuts_ctx* ctx, Run& r, cuts_mode mode) {
+    const int D = (int)ctx->part_depth;
+    const uint64_t sb0 = ctx->slice_begin, se0 = ctx->slice_end;
+    const uint32_t pt = ctx->part, np = ctx->nparts;
+    ctx->slice_begin = 0;
+    ctx->slice_end = ~0ull;
+    ctx->part = 0;
+    ctx->nparts = 1;
+    uint64_t n1 = 0;
+    const cuts_status s1 = build_level1(ctx, r, &n1);
+    ctx->slice_begin = sb0;
+    ctx->slice_end = se0;
+    ctx->part = pt;
+    ctx->nparts = np;
+    TRY(s1);
+    ctx->st.level_size[1] = n1;
+    if (n1) TRY(bfs_levels(ctx, r, 1, n1, D));
+    const uint64_t ND = ctx->st.level_size[D];
+    if (ctx->size_only) return read_ctrl(ctx);
+    uint64_t p0 = 0, cnt = 0;
+    slice_of(ctx, ND, &p0, &cnt);
+    uint64_t off;
+    TRY(alloc_bot(ctx, std::max<uint64_t>(cnt * D, 1) * sizeof(uint32_t), &off));
+    uint32_t* prows = (uint32_t*)(ctx->arena + off);
+    if (cnt) {
+        const Shuffle sh = make_shuffle(ctx->seed, ND);
+        const unsigned grid = (unsigned)std::min<uint64_t>((cnt + 255) / 256, (uint64_t)ctx->num_sms * 8);
+        switch (D) {
+            case 2: k_prefix_slice<2><<<grid, 256, 0, ctx->stream>>>(r.t, sh, p0, np, cnt, prows); break;
+            case 3: k_prefix_slice<3><<<grid, 256, 0, ctx->stream>>>(r.t, sh, p0, np, cnt, prows); break;
+            case 4: k_prefix_slice<4><<<grid, 256, 0, ctx->stream>>>(r.t, sh, p0, np, cnt, prows); break;
+            case 5: k_prefix_slice<5><<<grid, 256, 0, ctx->stream>>>(r.t, sh, p0, np, cnt, prows); break;
+            case 6: k_prefix_slice<6><<<grid, 256, 0, ctx->stream>>>(r.t, sh, p0, np, cnt, prows); break;
+            default: k_prefix_slice<7><<<grid, 256, 0, ctx->stream>>>(r.t, sh, p0, np, cnt, prows); break;
+        }
+        CK(cudaGetLastError());
+        ctx->st.launches++;
+    }
+    uint64_t upper[kMaxK + 1];
+    const bool first = std::min(sb0, ND) == 0 && pt == 0;
+    for (int l = 0; l <= kMaxK; ++l) upper[l] = (first && l < D) ? ctx->st.level_size[l] : 0;
+    TRY(build_prefix_levels(ctx, r, (uint32_t)D, cnt, prows));
+    for (int l = 1; l < D; ++l) ctx->st.level_size[l] = upper[l];
+    ctx->st.level_size[D] = cnt;
+    if (cnt) {
+        if (mode == CUTS_BFS) TRY(bfs_levels(ctx, r, D, cnt));
+        else TRY(hybrid_level(ctx, r, D, cnt));
+    }
+    return read_ctrl(ctx);
 }
 
 cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* rows, uint64_t cap_rows) {
@@ -1379,13 +1473,15 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
     const int k = (int)ctx->q.k;
     for (int j = 0; j <= kMaxK; ++j) { ctx->dfs_on[j] = false; ctx->dfs_next[j] = ctx->dfs_end[j] = 0; ctx->ord[j].valid = false; }
     if (ctx->pre_j) {
-        TRY(build_prefix_levels(ctx, r));
+        TRY(build_prefix_levels(ctx, r, ctx->pre_j, ctx->pre_count, ctx->pre_rows));
         const int J0 = (int)ctx->pre_j;
         if (ctx->pre_count > 0) {
             if (mode == CUTS_BFS) TRY(bfs_levels(ctx, r, J0, ctx->pre_count));
             else TRY(hybrid_level(ctx, r, J0, ctx->pre_count));
         }
         TRY(read_ctrl(ctx));
+    } else if (ctx->part_depth > 1 && (int)ctx->part_depth < k) {
+        TRY(partition_run(ctx, r, mode));
     } else {
     TRY(build_level1(ctx, r, &n1));
     ctx->st.level_size[1] = n1;
@@ -1676,6 +1772,29 @@ cuts_status cuts_set_root_slice(cuts_ctx* ctx, uint64_t begin, uint64_t end, uin
     ctx->slice_end = end;
     ctx->part = part;
     ctx->nparts = nparts;
+    return CUTS_OK;
+}
+
+cuts_status cuts_set_partition_depth(cuts_ctx* ctx, uint32_t depth) {
+    if (!ctx) return CUTS_EINVAL;
+    if (depth < 1 || depth >= (uint32_t)kMaxK) return fail(ctx, CUTS_EINVAL, "partition depth %u not in [1, %d)", depth, kMaxK);
+    ctx->part_depth = depth;
+    return CUTS_OK;
+}
+
+cuts_status cuts_partition_size(cuts_ctx* ctx, uint64_t* n) {
+    if (!ctx || !n) return CUTS_EINVAL;
+    if (!ctx->has_graph || !ctx->has_query) return fail(ctx, CUTS_ESTATE, "load_graph and set_query must precede cuts_partition_size");
+    const int k = (int)ctx->q.k;
+    if (ctx->part_depth <= 1 || (int)ctx->part_depth >= k) {
+        uint64_t nc = 0;
+        return cuts_level1_size(ctx, &nc, n);
+    }
+    ctx->size_only = true;
+    const cuts_status s = run_query(ctx, CUTS_HYBRID, false, nullptr, 0);
+    ctx->size_only = false;
+    TRY(s);
+    *n = ctx->st.level_size[ctx->part_depth];
     return CUTS_OK;
 }
 

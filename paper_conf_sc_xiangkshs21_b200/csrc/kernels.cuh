@@ -1804,6 +1804,27 @@ __global__ void k_prefix_export(Trie t, uint64_t e0, uint64_t cnt, uint32_t* __r
 }
 
 // lv[l] (l = 1..J) each hold cnt entries: (rows[i][l-1], i)
+// multi-GPU partition below level 1 (cuts_set_partition_depth): positions p0, p0 +
+// nparts, ... of the seeded shuffle of the whole level-J list, each exported as a flat
+// row of J vertices in matching-order positions (the seed format of cuts_set_prefixes)
+template <int J>
+__global__ void k_prefix_slice(Trie t, Shuffle sh, uint64_t p0, uint32_t nparts, uint64_t cnt,
+                               uint32_t* __restrict__ rows) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        uint2 cur = t.lv[J][sh.apply(p0 + i * nparts)];
+        uint32_t* row = rows + i * J;
+        row[J - 1] = cur.x;
+        uint32_t idx = cur.y;
+#pragma unroll
+        for (int p = J - 2; p >= 0; --p) {
+            cur = t.lv[p + 1][idx];
+            row[p] = cur.x;
+            idx = cur.y;
+        }
+    }
+}
+
 __global__ void k_prefix_import(const uint32_t* __restrict__ rows, uint32_t J, uint64_t cnt, Trie t) {
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt;
          i += (uint64_t)gridDim.x * blockDim.x) {

@@ -98,3 +98,42 @@ def test_world2_through_the_abi_one_gpu(cuts):
         locals_ = [results[r][1][q.name][0] for r in range(2)]
         assert sum(locals_) == want
         assert all(results[r][1][q.name][1] == want for r in range(2))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("depth", [1, 2, 3])
+def test_partition_depth_parts_sum_to_oracle(depth):
+    """cuts_set_partition_depth: the cyclic parts (and chunked slices) of the shuffled
+    level-D list sum to the oracle count, and their level sizes to the oracle's, in
+    HYBRID and BFS, on the DLR (K6), local-rows (K5) and windowed (K5-P3, C4) paths."""
+    import oracle
+    from inputs import rmat_graph, named_query, DENSE5, dense_family
+    from paper_conf_sc_xiangkshs21_b200 import Cuts
+    g = rmat_graph(9, 8, 0.50, 0.20, 0.20, seed=3)
+    c = Cuts(device=0, arena_bytes=512 << 20)
+    c.load_csr(g)
+    for q in (dense_family(6)[0], DENSE5[0], DENSE5[2], named_query("C4")):
+        want, lv = oracle.count(g, q, levels=True)
+        qr, qc = q.csr()
+        c.set_query(qr, qc)
+        c.set_partition_depth(depth)
+        L = c.partition_size()
+        assert L == lv[min(depth, q.k - 1) if depth < q.k else 1]
+        for nparts in (1, 3):
+            for mode in ("hybrid", "bfs"):
+                tot, lvs = 0, [0] * (q.k + 1)
+                for part in range(nparts):
+                    c.set_root_slice(0, 2**64 - 1, part, nparts)
+                    tot += c.count(mode)
+                    for j, v in enumerate(c.stats()["level_size"]):
+                        lvs[j] += v
+                assert tot == want, (q.name, depth, nparts, mode)
+                assert lvs == lv, (q.name, depth, nparts, mode)
+        tot = 0                                      # chunks of the shuffled list (the dynamic queue's unit)
+        for b in range(0, L, max(1, L // 4)):
+            c.set_root_slice(b, b + max(1, L // 4), 0, 1)
+            tot += c.count("hybrid")
+        assert tot == want, (q.name, depth, "chunks")
+        c.set_root_slice(0, 2**64 - 1, 0, 1)
+    c.set_partition_depth(1)
+    c.close()
