@@ -147,6 +147,8 @@ typedef struct {
 #define CUTS_DEBUG_TAIL_ALT 8192u /* ablation: the deep-local-rows tail gives one lane per
                                   triangle (warp scan + shuffle search) instead of one lane
                                   per level-(k-2) entry                                     */
+#define CUTS_DEBUG_TAIL_SPLIT 16384u /* experiment: the tail queues entries split into
+                                  work items of 8 triangles                                 */
 #define CUTS_DEBUG_GROUPS 2048u /* instrumentation: histogram of sibling-group sizes (children
                                   per entry) of every ordered level, read with
                                   cuts_debug_group_hist                                     */

@@ -60,6 +60,8 @@ struct cuts_ctx {
     uint32_t* deg = nullptr;
     uint32_t* hub = nullptr;               // hub[v] -> bitmap row, or kNoHub
     uint32_t* bm = nullptr;                // hub bitmaps
+    uint32_t* cb = nullptr;                // hub-to-hub core bitmap (nhubs^2 bits)
+    uint32_t cbw = 0;
     uint32_t* colx = nullptr;              // packed (id | min(deg,31) << 27) copy of col, or null
     uint32_t words = 0;
     uint64_t nhubs = 0, hub_t_used = 0;
@@ -979,7 +981,9 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
             int tm = -1;
             if (timing) { tm = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[tm], ctx->stream)); }
             const unsigned gt = (unsigned)std::min<uint64_t>((size + 255) / 256, (uint64_t)ctx->num_sms * 16);
-            auto kt = cb ? k_dlr_tail<true, 0> : ((ctx->debug & CUTS_DEBUG_TAIL_ALT) ? k_dlr_tail<false, 1> : k_dlr_tail<false, 0>);
+            auto kt = cb ? k_dlr_tail<true, 0>
+                          : ((ctx->debug & CUTS_DEBUG_TAIL_ALT) ? k_dlr_tail<false, 1>
+                             : ((ctx->debug & CUTS_DEBUG_TAIL_SPLIT) ? k_dlr_tail<false, 2> : k_dlr_tail<false, 0>));
             kt<<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
                                             (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
             CK(cudaGetLastError());
@@ -1173,6 +1177,7 @@ cuts_status build_hubs(cuts_ctx* ctx) {
     ctx->hub_t_used = 0;
     ctx->hub = nullptr;
     ctx->bm = nullptr;
+    ctx->cb = nullptr;
     if (ctx->hub_t == 0xFFFFFFFFu || ctx->n == 0 || ctx->nnz == 0) return CUTS_OK;
     const uint32_t n = ctx->n;
     ctx->words = (n + 31) / 32;
@@ -1208,13 +1213,21 @@ cuts_status build_hubs(cuts_ctx* ctx) {
     }
     ctx->bm = (uint32_t*)(ctx->arena + ctx->base_off + hub_bytes);
     CK(cudaMemsetAsync(ctx->bm, 0, nh * row_bytes, ctx->stream));
+    // core bitmap: hub x hub adjacency in hub-row coordinates, when it is small (<= 64 MB)
+    ctx->cb = nullptr;
+    ctx->cbw = (uint32_t)((nh + 31) / 32);
+    const uint64_t cb_bytes = align_up(nh * (uint64_t)ctx->cbw * 4);
+    if (cb_bytes <= (64ull << 20) && ctx->base_off + hub_bytes + bm_bytes + cb_bytes + (64u << 10) <= ctx->arena_bytes) {
+        ctx->cb = (uint32_t*)(ctx->arena + ctx->base_off + hub_bytes + bm_bytes);
+        CK(cudaMemsetAsync(ctx->cb, 0, cb_bytes, ctx->stream));
+    }
     unsigned g2 = (unsigned)std::min<uint64_t>(((uint64_t)n * 32 + 255) / 256, (uint64_t)ctx->num_sms * 16);
-    k_hub_fill<<<g2, 256, 0, ctx->stream>>>(ctx->row_ptr, ctx->col, n, ctx->hub, ctx->words, ctx->bm);
+    k_hub_fill<<<g2, 256, 0, ctx->stream>>>(ctx->row_ptr, ctx->col, n, ctx->hub, ctx->words, ctx->bm, ctx->cb, ctx->cbw);
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(ctx->stream));
     ctx->nhubs = nh;
     ctx->hub_t_used = t;
-    ctx->base_off += hub_bytes + bm_bytes;
+    ctx->base_off += hub_bytes + bm_bytes + (ctx->cb ? cb_bytes : 0);
     return CUTS_OK;
 }
 
@@ -1451,6 +1464,7 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
         return fail(ctx, CUTS_EINVAL, "%s query on a %s graph", ctx->q_directed ? "directed" : "undirected",
                     ctx->directed ? "directed" : "undirected");
     r.g = Graph{ctx->row_ptr, ctx->col, ctx->deg, ctx->nhubs ? ctx->hub : nullptr, ctx->bm, ctx->n, ctx->words, ctx->colx};
+    if (ctx->nhubs && ctx->cb) { r.g.cb = ctx->cb; r.g.cbw = ctx->cbw; }
     r.g.dn = ctx->directed ? ctx->n : 0u;
     ctx->q.src_first = (ctx->debug & CUTS_DEBUG_FIRST_SOURCE) ? 1u : 0u;
     ctx->q.count_fast = (!enumerate && !(ctx->debug & (CUTS_DEBUG_NO_FAST_COUNT | CUTS_DEBUG_SV))) ? 1u : 0u;

@@ -102,7 +102,21 @@ struct Graph {
     const uint32_t* __restrict__ colx;  // col with min(deg, 31) packed in bits 27..31 (nullptr: n >= 2^27)
     const uint32_t* __restrict__ fre = nullptr;   // free lists of component roots (QPlan::foff/flen)
     uint32_t dn = 0;   // directed: rows [0,n) are out-lists, rows [n,2n) in-lists, dn = n; undirected: 0
+    // hub-to-hub core bitmap: row h (a hub) has bit hub[u] set for every hub neighbour u —
+    // nhubs^2 bits (32 MB at 16 K hubs), small enough to stay in L2 (nullptr: none)
+    const uint32_t* __restrict__ cb = nullptr;
+    uint32_t cbw = 0;  // u32 words per core row
 };
+
+// is c in N(v) for a hub v with bitmap row h: the L2-resident core row when c is a hub
+// too, else the full n-bit row
+__device__ __forceinline__ bool hub_probe(const Graph& g, uint32_t h, uint32_t c) {
+    if (g.cb) {
+        const uint32_t hc = __ldg(g.hub + c);
+        if (hc != 0xffffffffu) return (__ldg(g.cb + (uint64_t)h * g.cbw + (hc >> 5)) >> (hc & 31)) & 1u;
+    }
+    return (__ldg(g.bm + (uint64_t)h * g.words + (c >> 5)) >> (c & 31)) & 1u;
+}
 
 constexpr uint32_t kNoHub = 0xffffffffu;
 constexpr int kPackShift = 27;               // colx: vertex id in bits 0..26, min(deg, 31) above
@@ -189,7 +203,8 @@ __global__ void k_hub_mark(const uint32_t* __restrict__ deg, uint32_t n, uint32_
 
 // one warp per vertex: hubs set the bits of their neighbours
 __global__ void k_hub_fill(const uint64_t* __restrict__ row_ptr, const uint32_t* __restrict__ col, uint32_t n,
-                           const uint32_t* __restrict__ hub, uint32_t words, uint32_t* __restrict__ bm) {
+                           const uint32_t* __restrict__ hub, uint32_t words, uint32_t* __restrict__ bm,
+                           uint32_t* __restrict__ cb, uint32_t cbw) {
     const int lane = threadIdx.x & 31;
     const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
@@ -200,6 +215,10 @@ __global__ void k_hub_fill(const uint64_t* __restrict__ row_ptr, const uint32_t*
         for (uint64_t p = row_ptr[v] + lane; p < row_ptr[v + 1]; p += 32) {
             const uint32_t u = col[p];
             atomicOr(row + (u >> 5), 1u << (u & 31));
+            if (cb) {
+                const uint32_t hu = hub[u];
+                if (hu != kNoHub) atomicOr(cb + (uint64_t)h * cbw + (hu >> 5), 1u << (hu & 31));
+            }
         }
     }
 }
@@ -1235,6 +1254,7 @@ __global__ void __launch_bounds__(256, 6) k_dlr_rows(Graph g, Dlr a, unsigned lo
             uint64_t g0 = 0, rb = 0;
             const uint32_t* lb = g.col;
             bool bmp = false;
+            uint32_t hrow = 0;
             if (has) {
                 const DlrGrp gr = dlr_group(a, e);
                 g0 = gr.g0; m = gr.m; W = gr.W; rb = gr.rb;
@@ -1246,7 +1266,7 @@ __global__ void __launch_bounds__(256, 6) k_dlr_rows(Graph g, Dlr a, unsigned lo
                     const uint32_t h = g.hub ? __ldg(g.hub + v) : kNoHub;
                     if (h != kNoHub) {
                         bmp = true;
-                        lb = g.bm + (uint64_t)h * g.words;
+                        hrow = h;
                     } else {
                         const uint64_t b = g.row_ptr[v];
                         lb = g.col + b;
@@ -1268,7 +1288,7 @@ __global__ void __launch_bounds__(256, 6) k_dlr_rows(Graph g, Dlr a, unsigned lo
                 const uint32_t c = act ? a.lv[g0 + jj].x : 0u;
                 bool ok = act;
                 if (count_bytes && act) b_need += 4ull + 4ull * (bmp ? 1u : (32u - __clz(len)));
-                if (bmp && act) ok = (__ldg(lb + (c >> 5)) >> (c & 31)) & 1u;
+                if (bmp && act) ok = hub_probe(g, hrow, c);
                 const bool pend = act && !bmp;
                 const unsigned pw = __ballot_sync(0xffffffffu, pend);
                 uint32_t pos = 0;
@@ -1442,6 +1462,75 @@ __device__ __forceinline__ uint32_t dlr_fns64(unsigned long long y, uint32_t ran
     return rank < plo ? (uint32_t)__fns(lo, 0, (int)rank + 1) : 32u + (uint32_t)__fns((uint32_t)(y >> 32), 0, (int)(rank - plo) + 1);
 }
 
+// Members l of x = A_t & A_s & {> s} with ranks [r0, r0 + kDlrRun) in ascending order (fewer
+// if x runs out): k4 += |x & {> l} & A_l| for each — one split work item of the tail.
+// WM: x in registers for rows of up to WM words (0: re-read from the rows).
+constexpr uint32_t kDlrRun = 8;
+template <int WM>
+__device__ __forceinline__ void dlr_run(const unsigned long long* __restrict__ Rg, uint32_t te, uint32_t s, uint32_t W,
+                                        uint32_t r0, unsigned long long& k4) {
+    const unsigned long long* Rt = Rg + (uint64_t)te * W;
+    const unsigned long long* Rs = Rg + (uint64_t)s * W;
+    uint32_t rem = kDlrRun, skip = r0;
+    if constexpr (WM > 0) {
+        unsigned long long x[WM];
+#pragma unroll
+        for (int w = 0; w < WM; ++w) x[w] = (uint32_t)w < W ? (Rt[w] & Rs[w] & dlr_above(s, (uint32_t)w)) : 0ull;
+#pragma unroll
+        for (int w = 0; w < WM; ++w) {
+            unsigned long long y = x[w];
+            const uint32_t pc = (uint32_t)__popcll(y);
+            if (rem == 0 || skip >= pc) { skip -= min(skip, pc); continue; }
+            if (skip) {                                       // drop the members of lower rank
+                const uint32_t p = dlr_fns64(y, skip - 1);
+                y &= p == 63u ? 0ull : (~0ull << (p + 1u));
+                skip = 0;
+            }
+            while (y && rem) {
+                const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                y &= y - 1;                                   // x's members above l in word w
+                --rem;
+                const unsigned long long* Rl = Rg + (uint64_t)l * W;
+                unsigned long long c = __popcll(y & Rl[w]);
+#pragma unroll
+                for (int v = w + 1; v < WM; ++v) c += (uint32_t)v < W ? __popcll(x[v] & Rl[v]) : 0ull;
+                k4 += c;
+            }
+        }
+    } else {
+        for (uint32_t w = s >> 6; w < W && rem; ++w) {
+            unsigned long long y = Rt[w] & Rs[w] & dlr_above(s, w);
+            const uint32_t pc = (uint32_t)__popcll(y);
+            if (skip >= pc) { skip -= pc; continue; }
+            if (skip) {
+                const uint32_t p = dlr_fns64(y, skip - 1);
+                y &= p == 63u ? 0ull : (~0ull << (p + 1u));
+                skip = 0;
+            }
+            while (y && rem) {
+                const uint32_t l = 64u * w + (uint32_t)(__ffsll((long long)y) - 1);
+                y &= y - 1;
+                --rem;
+                const unsigned long long* Rl = Rg + (uint64_t)l * W;
+                unsigned long long c = __popcll(y & Rl[w]);
+                for (uint32_t v = w + 1; v < W; ++v) c += __popcll(Rt[v] & Rs[v] & Rl[v]);
+                k4 += c;
+            }
+        }
+    }
+}
+
+// a split work item: te (10 bits) | s (10) | W - 1 (4) | run index j (8) -> ranks [8j, 8j+8)
+__device__ __forceinline__ void dlr_split_item(const unsigned long long* __restrict__ R, unsigned long long rb, uint32_t pk,
+                                               unsigned long long& k4) {
+    const uint32_t te = pk & 0x3ffu, s = (pk >> 10) & 0x3ffu, W = ((pk >> 20) & 0xfu) + 1u, r0 = (pk >> 24) * kDlrRun;
+    const unsigned long long* Rg = R + rb;
+    if (W == 1) dlr_run<1>(Rg, te, s, 1, r0, k4);
+    else if (W == 2) dlr_run<2>(Rg, te, s, 2, r0, k4);
+    else if (W <= 4) dlr_run<4>(Rg, te, s, W, r0, k4);
+    else dlr_run<0>(Rg, te, s, W, r0, k4);
+}
+
 // CUTS_DEBUG_TAIL_ALT (ablation): drain the 32 queued entries with one lane per
 // triangle instead of one lane per entry — each entry's x (rows of <= 4 words) is staged in
 // the warp's shared memory, a warp scan numbers the triangles, every round gives each lane
@@ -1529,7 +1618,7 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
                                                   uint32_t lev1, uint32_t bw1, uint32_t bw2) {
     __shared__ unsigned long long q_rb[8][64];
     __shared__ uint32_t q_pk[8][64];
-    __shared__ unsigned long long q_x[V ? 8 : 1][V ? 128 : 1];   // CUTS_DEBUG_TAIL_ALT: staged x words
+    __shared__ unsigned long long q_x[V == 1 ? 8 : 1][V == 1 ? 128 : 1];   // CUTS_DEBUG_TAIL_ALT: staged x words
     unsigned long long tri = 0, k4 = 0, b_plan = 0, b_ext = 0, b_out = 0, b_need = 0, b_ops = 0;
     const uint64_t c0 = cpos_b[e0];
     const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
@@ -1579,6 +1668,37 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
                 }
             }
         }
+        if (V == 2) {
+            // split work items: an entry with |x| = n becomes ceil(n / kDlrRun) queue items
+            uint32_t n = 0;
+            if (up) {
+                const uint32_t te = pk & 0x7ffu, s = (pk >> 11) & 0x7ffu, W = pk >> 22;
+                const unsigned long long* Rt = a.R + rb + (uint64_t)te * W;
+                const unsigned long long* Rs = a.R + rb + (uint64_t)s * W;
+                for (uint32_t w = s >> 6; w < W; ++w) n += (uint32_t)__popcll(Rt[w] & Rs[w] & dlr_above(s, w));
+                tri += n;
+                pk = te | (s << 10) | ((W - 1) << 20);
+            }
+            const uint32_t nsub = (n + kDlrRun - 1) / kDlrRun;
+            for (uint32_t j = 0;; ++j) {
+                const bool want = j < nsub;
+                const unsigned bj = __ballot_sync(0xffffffffu, want);
+                if (!bj) break;
+                if (want) {
+                    const uint32_t pos = qn + __popc(bj & ((1u << lane) - 1u));
+                    q_rb[wq][pos] = rb;
+                    q_pk[wq][pos] = pk | (j << 24);
+                }
+                qn += __popc(bj);
+                __syncwarp();
+                if (qn >= 32) {
+                    dlr_split_item(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], k4);
+                    qn -= 32;
+                    __syncwarp();
+                }
+            }
+            continue;
+        }
         const unsigned bal = __ballot_sync(0xffffffffu, up);
         if (up) {
             const uint32_t pos = qn + __popc(bal & ((1u << lane) - 1u));
@@ -1588,15 +1708,17 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
         qn += __popc(bal);
         __syncwarp();
         if (qn >= 32) {                                     // drain the 32 newest items
-            if (V) dlr_drain_tri(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], true, q_x[V ? wq : 0], tri, k4);
+            if (V == 1) dlr_drain_tri(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], true, q_x[V == 1 ? wq : 0], tri, k4);
             else dlr_tail_item(a.R, q_rb[wq][qn - 32 + lane], q_pk[wq][qn - 32 + lane], tri, k4);
             qn -= 32;
             __syncwarp();
         }
     }
-    if (V) {
+    if (V == 2) {
+        if ((uint32_t)lane < qn) dlr_split_item(a.R, q_rb[wq][lane], q_pk[wq][lane], k4);
+    } else if (V) {
         if (qn) dlr_drain_tri(a.R, (uint32_t)lane < qn ? q_rb[wq][lane] : 0ull, (uint32_t)lane < qn ? q_pk[wq][lane] : 0u,
-                              (uint32_t)lane < qn, q_x[V ? wq : 0], tri, k4);
+                              (uint32_t)lane < qn, q_x[V == 1 ? wq : 0], tri, k4);
     } else if ((uint32_t)lane < qn) {
         dlr_tail_item(a.R, q_rb[wq][lane], q_pk[wq][lane], tri, k4);
     }
