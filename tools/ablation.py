@@ -12,7 +12,10 @@ k_extend milliseconds.  Variants (all give the same counts; checked here):
   packed    : + packed (id | degree) stream (degree filter without a gather)
   reuse     : + ancestor-set source
   fastcount : + set-difference count at a single-list degree-free last level
-  full      : + pair-shared symmetric last level (the product default)
+  pairs     : + pair-shared symmetric last level
+  lr        : + local rows of the level-(k-2) sibling groups (round 1)
+  full      : + deep local rows of the level-(k-3) groups and the symmetric tail
+              (round 2; the product default)
 Side variants (NEXT-2, compare with the chain member named):
   binned    : fastcount with binned virtual warps at the last level
               instead of the single bin
@@ -40,6 +43,8 @@ VARIANTS = [  # (name, hub threshold, debug kwargs)
     ("packed", 0, dict(no_reuse=True, no_fast_count=True)),
     ("reuse", 0, dict(no_fast_count=True, no_pairs=True)),
     ("fastcount", 0, dict(no_pairs=True)),
+    ("pairs", 0, dict(no_lr=True)),
+    ("lr", 0, dict(no_dlr=True)),
     ("full", 0, dict()),
     ("binned", 0, dict(no_pairs=True, binned=True)),
     ("sv", None, dict(sv=True)),
@@ -53,6 +58,7 @@ def main():
     ap.add_argument("--variants", default=",".join(v[0] for v in VARIANTS))
     ap.add_argument("--query", default="")
     ap.add_argument("--out", default="")
+    ap.add_argument("--range", default="", help="override the workload's root range: absolute canonical a:b")
     args = ap.parse_args()
     wl = WORKLOADS[args.workload]
     ctx = Cuts(device=0)
@@ -76,7 +82,9 @@ def main():
                 best, st, c = None, None, None
                 for _ in range(args.reps):
                     ctx.set_query(qr, qc)
-                    if wl.root_range is not None:
+                    if args.range:
+                        ctx.set_root_range(*(int(x) for x in args.range.split(":")))
+                    elif wl.root_range is not None:
                         ctx.set_root_range(*wl.roots(ctx.level1_size()[0]))
                     torch.cuda.synchronize()
                     t = time.time()
@@ -87,7 +95,8 @@ def main():
                 key = (spec.name, q.name)
                 assert want.setdefault(key, c) == c, (name, key, c, want[key])
                 totals[name] += best
-                rec = {"variant": name, "graph": spec.name, "query": q.name, "count": c, "s": round(best, 4),
+                rec = {"variant": name, "graph": spec.name, "query": q.name, "range": args.range or None,
+                       "count": c, "s": round(best, 4),
                        "ms_extend": round(st["ms_extend"], 2), "ms_plan": round(st["ms_plan"], 2),
                        "hubs": st["hubs"], "items": st["items"]}
                 line = json.dumps(rec)
