@@ -149,6 +149,9 @@ typedef struct {
                                   per level-(k-2) entry                                     */
 #define CUTS_DEBUG_TAIL_SPLIT 16384u /* experiment: the tail queues entries split into
                                   work items of 8 triangles                                 */
+#define CUTS_DEBUG_NO_CTA_TAIL 32768u /* ablation: the deep-rows tail of wide-row groups
+                                  (W >= 2) stays in the warp-queue kernel instead of a CTA per
+                                  group with its rows staged in shared memory by TMA        */
 #define CUTS_DEBUG_GROUPS 2048u /* instrumentation: histogram of sibling-group sizes (children
                                   per entry) of every ordered level, read with
                                   cuts_debug_group_hist                                     */

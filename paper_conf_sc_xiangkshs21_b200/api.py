@@ -281,14 +281,16 @@ class Cuts:
                   no_pack: bool = False, first_source: bool = False, no_fast_count: bool = False,
                   preload_count: bool = False, binned: bool = False, sv: bool = False, no_pairs: bool = False,
                   no_lr: bool = False, groups: bool = False, no_dlr: bool = False,
-                  tail_alt: bool = False, tail_split: bool = False):
+                  tail_alt: bool = False, tail_split: bool = False,
+                  no_cta_tail: bool = False):
         """CUTS_DEBUG_* flags: instrumentation and the NEXT-2 ablations (include/cuts.h)."""
         flags = ((1 if timing else 0) | (2 if bytes_ else 0) | (4 if no_reuse else 0) |
                  (8 if no_pack else 0) | (16 if first_source else 0) | (32 if no_fast_count else 0) |
                  (64 if preload_count else 0) | (128 if binned else 0) | (256 if sv else 0) |
                  (512 if no_pairs else 0) | (1024 if no_lr else 0) | (2048 if groups else 0) |
                  (4096 if no_dlr else 0) | (8192 if tail_alt else 0) |
-                 (16384 if tail_split else 0))
+                 (16384 if tail_split else 0) |
+                 (32768 if no_cta_tail else 0))
         self._check(self.lib.cuts_set_debug(self.h, flags))
         return self
 

@@ -932,6 +932,23 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
     CK(cudaMemsetAsync(a.R, 0, words * 8, ctx->stream));
     k_dlr_desc<<<(unsigned)std::min<uint64_t>((N + 255) / 256, (uint64_t)ctx->num_sms * 16), 256, 0, ctx->stream>>>(a);
     CK(cudaGetLastError());
+    // the W >= 2 groups, ascending by parent slot: k_dlr_tail_cta's work list
+    const bool cta_tail = !cb && !(ctx->debug & (CUTS_DEBUG_TAIL_ALT | CUTS_DEBUG_TAIL_SPLIT | CUTS_DEBUG_NO_CTA_TAIL));
+    DlrWide wide{nullptr, 0};
+    if (cta_tail) {
+        thrust::counting_iterator<uint32_t> it(0);
+        const DlrIsWide pred{o.cpos, o.ea};
+        size_t sel_bytes = 0;
+        CK(cub::DeviceSelect::If(nullptr, sel_bytes, it, (uint32_t*)nullptr, ctx->ctrl + kNumSel, (int64_t)ng, pred, ctx->stream));
+        uint64_t woff;
+        TRY(alloc_top(ctx, align_up(std::max<uint64_t>(ng, 1) * 4) + align_up(sel_bytes), &woff));
+        uint32_t* wl = (uint32_t*)(ctx->arena + woff);
+        CK(cub::DeviceSelect::If(ctx->arena + woff + align_up(std::max<uint64_t>(ng, 1) * 4), sel_bytes, it, wl,
+                                 ctx->ctrl + kNumSel, (int64_t)ng, pred, ctx->stream));
+        CK(cudaMemcpyAsync(ctx->h_ctrl + kNumSel, ctx->ctrl + kNumSel, 8, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        wide = DlrWide{wl, (uint32_t)ctx->h_ctrl[kNumSel]};
+    }
     const double avg = (double)N / (double)std::max<uint64_t>(ng, 1) / 2;     // members tested per entry
     auto go = [&](auto kern, int G) {
         static int occ[4] = {0, 0, 0, 0};
@@ -968,6 +985,14 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
         ctx->st.launches++;
         const uint64_t eb = ctx->h_ctrl[kFind], size = ctx->h_ctrl[kFind + 1];
         if (eb <= ea) return fail(ctx, CUTS_ENOMEM, "HYBRID: one level-%d entry's children exceed the arena share", J);
+        uint32_t xa = 0, xb = 0;                  // parent slots of the chunk's first and last level-J entry
+        if (wide.n && size) {
+            CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 2, &a.lv[ea], 8, cudaMemcpyDeviceToHost, ctx->stream));
+            CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 3, &a.lv[eb - 1], 8, cudaMemcpyDeviceToHost, ctx->stream));
+            CK(cudaStreamSynchronize(ctx->stream));
+            xa = (uint32_t)((ctx->h_ctrl[kCtrlWords + 2] >> 32) - o.w0 - o.ea);
+            xb = (uint32_t)((ctx->h_ctrl[kCtrlWords + 3] >> 32) - o.w0 - o.ea);
+        }
         if (size) {
             const uint64_t bot_save = ctx->bot;
             TRY(alloc_bot(ctx, size * sizeof(uint2), &off));
@@ -983,9 +1008,22 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
             const unsigned gt = (unsigned)std::min<uint64_t>((size + 255) / 256, (uint64_t)ctx->num_sms * 16);
             auto kt = cb ? k_dlr_tail<true, 0>
                           : ((ctx->debug & CUTS_DEBUG_TAIL_ALT) ? k_dlr_tail<false, 1>
-                             : ((ctx->debug & CUTS_DEBUG_TAIL_SPLIT) ? k_dlr_tail<false, 2> : k_dlr_tail<false, 0>));
+                             : ((ctx->debug & CUTS_DEBUG_TAIL_SPLIT) ? k_dlr_tail<false, 2>
+                                : (wide.n ? k_dlr_tail<false, 3> : k_dlr_tail<false, 0>)));
             kt<<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
                                             (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            if (wide.n) {   // the W >= 2 groups: a CTA per group, rows staged by TMA
+                static int occ = 0;
+                if (!occ) {
+                    cudaFuncSetAttribute(k_dlr_tail_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kDlrSmemBytes);
+                    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dlr_tail_cta, 256, kDlrSmemBytes);
+                    if (occ < 1) occ = 1;
+                }
+                CK(cudaMemsetAsync(ctx->ctrl + kDlrWork, 0, sizeof(unsigned long long), ctx->stream));
+                k_dlr_tail_cta<<<(unsigned)(ctx->num_sms * occ), 256, kDlrSmemBytes, ctx->stream>>>(
+                    a, cposb, ea, eb, out, ctx->ctrl, wide, xa, xb);
+                ctx->st.launches++;
+            }
             CK(cudaGetLastError());
             if (timing) {
                 const int t1 = next_event(ctx);

@@ -24,7 +24,8 @@ constexpr int kMaxK = 8;
 constexpr int kLrMaxM = 512;                // local rows: largest sibling group held in shared memory
 constexpr int kLrWords = kLrMaxM / 32;
 constexpr int kLrBatch = 256;
-constexpr int kDlrMaxM = 1024;             // deep local rows: largest sibling group (16 u64 words per row)              // k_lr_group: parent slots claimed per CTA fetch
+constexpr int kDlrMaxM = 1024;
+constexpr uint32_t kDlrSmemBytes = 64u << 10;   // k_dlr_tail_cta: rows staged per group (W >= 2 groups up to this)             // deep local rows: largest sibling group (16 u64 words per row)              // k_lr_group: parent slots claimed per CTA fetch
 constexpr int kTile = 256;   // items per CTA tile == threads per CTA
 
 struct QPlan {                 // query in matching-order positions
@@ -1212,6 +1213,16 @@ __global__ void k_dlr_desc(Dlr a) {
     }
 }
 
+// CUB select predicate: parent slot x (window-relative, from ea) owns a group with W >= 2
+struct DlrIsWide {
+    const uint64_t* cpos;
+    uint64_t ea;
+    __host__ __device__ bool operator()(const uint32_t& x) const {
+        const uint64_t m = cpos[ea + x + 1] - cpos[ea + x];
+        return m > 64 && m <= (uint64_t)kDlrMaxM;
+    }
+};
+
 // per parent slot: row words of its group (0 when it is left to the windowed pipeline)
 __global__ void k_dlr_layout(Dlr a, uint64_t* __restrict__ rw, unsigned long long* __restrict__ ctrl) {
     unsigned long long large = 0;
@@ -1219,7 +1230,7 @@ __global__ void k_dlr_layout(Dlr a, uint64_t* __restrict__ rw, unsigned long lon
     for (uint64_t x = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; x <= ng; x += (uint64_t)gridDim.x * blockDim.x) {
         if (x == ng) { rw[ng] = 0; continue; }
         const uint64_t m = a.cpos[a.ea + x + 1] - a.cpos[a.ea + x];
-        rw[x] = m <= (uint64_t)kDlrMaxM ? m * ((m + 63) / 64) : 0ull;
+        rw[x] = m <= (uint64_t)kDlrMaxM ? ((m * ((m + 63) / 64) + 1) & ~1ull) : 0ull;   // even: 16-B aligned blocks
         if (m > (uint64_t)kDlrMaxM) large += m;
     }
     large = warp_sum(large);
@@ -1634,8 +1645,9 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
             const DlrGrp gr = dlr_group(a, e);
             const uint32_t te = (uint32_t)(e - gr.g0);
             const unsigned long long* Rt = a.R + gr.rb + (uint64_t)te * gr.W;
-            const uint32_t s = dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0)));
-            up = te < s;
+            const bool mine = !(V == 3 && gr.W >= 2);          // V 3: k_dlr_tail_cta takes W >= 2
+            const uint32_t s = mine ? dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0))) : 0u;
+            up = mine && te < s;
             rb = gr.rb;
             pk = te | (s << 11) | (gr.W << 22);
             if (count_bytes) {
@@ -1732,6 +1744,129 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
         flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
         b_ops = warp_sum(b_ops);
         if (lane == 0 && b_ops) atomicAdd(ctrl + kTailOps, b_ops);
+    }
+}
+
+// ---- the tail for wide-row groups: one CTA per group, the rows staged by TMA ----------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+// Groups with W >= 2 (more than 64 members) hold most of the tail's work and reuse their
+// m x W row block across all their level-(b+1) entries: a CTA takes one such group at a
+// time (dynamic queue over the chunk's parent slots), one elected thread stages the
+// block into shared memory with a single bulk copy (cp.async.bulk, completion on an
+// mbarrier; blocks above kDlrSmemBytes stay in global memory), and the warps run the
+// warp-queue algebra of k_dlr_tail over the group's stored entries with the rows read
+// from shared memory.  Entries of W = 1 groups are left to k_dlr_tail (skip_narrow).
+struct DlrWide {                      // parent slots (x = q - ea) of the W >= 2 groups, ascending (DlrIsWide)
+    const uint32_t* __restrict__ x;
+    uint32_t n;
+};
+
+__global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0,
+                                                      uint64_t e1, const uint2* __restrict__ out,
+                                                      unsigned long long* __restrict__ ctrl, DlrWide wide,
+                                                      uint32_t xa, uint32_t xb) {
+    extern __shared__ __align__(16) unsigned long long srow[];
+    __shared__ __align__(8) unsigned long long mbar;
+    __shared__ uint32_t q_pk[8][64];
+    __shared__ uint64_t s_q;
+    unsigned long long tri = 0, k4 = 0;
+    const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
+    const uint64_t c0 = cpos_b[e0], cbase = a.cpos[a.ea];
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar)));
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    __syncthreads();
+    uint32_t phase = 0;
+    // the wide groups whose slots lie in [xa, xb] (the level-b entries of this chunk)
+    uint32_t lo = 0, hi = wide.n;
+    {
+        uint32_t l = 0, h = wide.n;
+        while (l < h) { const uint32_t mid = (l + h) / 2; if (wide.x[mid] < xa) l = mid + 1; else h = mid; }
+        lo = l;
+        h = wide.n;
+        while (l < h) { const uint32_t mid = (l + h) / 2; if (wide.x[mid] <= xb) l = mid + 1; else h = mid; }
+        hi = l;
+    }
+    for (;;) {
+        if (threadIdx.x == 0) s_q = lo + atomicAdd(ctrl + kDlrWork, 1ull);
+        __syncthreads();
+        if (s_q >= hi) break;
+        const uint64_t q = a.ea + wide.x[s_q];
+        const uint64_t g0 = a.cpos[q] - cbase;
+        const uint32_t m = (uint32_t)(a.cpos[q + 1] - a.cpos[q]);
+        const uint32_t W = (m + 63) / 64;
+        if (W < 2 || m > (uint32_t)kDlrMaxM) { __syncthreads(); continue; }
+        const uint64_t t0 = g0 > e0 ? g0 : e0, t1 = (g0 + m < e1) ? g0 + m : e1;
+        if (t0 >= t1) { __syncthreads(); continue; }
+        const uint64_t F0 = cpos_b[t0] - c0, F1 = cpos_b[t1] - c0;
+        const unsigned long long rb = a.roff[q - a.ea];
+        const uint32_t bytes = (uint32_t)((((uint64_t)m * W + 1) & ~1ull) * 8);
+        const bool staged = bytes <= kDlrSmemBytes;
+        if (staged) {
+            if (threadIdx.x == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // earlier generic reads of srow
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
+                             ::"r"(smem_u32(&mbar)), "r"(bytes) : "memory");
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(smem_u32(srow)), "l"(a.R + rb), "r"(bytes), "r"(smem_u32(&mbar)) : "memory");
+            }
+            uint32_t done = 0;
+            while (!done) {
+                asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+                             : "=r"(done) : "r"(smem_u32(&mbar)), "r"(phase) : "memory");
+            }
+            phase ^= 1u;
+        }
+        const unsigned long long* Rg = staged ? srow : a.R + rb;
+        uint32_t qn = 0;
+        for (uint64_t base = F0 + (uint64_t)wq * 32; base < F1; base += 256) {
+            const uint64_t f = base + lane;
+            bool up = false;
+            uint32_t pk = 0;
+            if (f < F1) {
+                const uint32_t e = out[f].y;
+                const uint32_t te = (uint32_t)(e - g0);
+                const uint32_t s = dlr_select(Rg + (uint64_t)te * W, W, (uint32_t)(f - (cpos_b[e] - c0)));
+                up = te < s;
+                pk = te | (s << 11) | (W << 22);
+            }
+            const unsigned bal = __ballot_sync(0xffffffffu, up);
+            if (up) {
+                const uint32_t pos = qn + __popc(bal & ((1u << lane) - 1u));
+                q_pk[wq][pos] = pk;
+            }
+            qn += __popc(bal);
+            __syncwarp();
+            if (qn >= 32) {
+                const uint32_t pq = q_pk[wq][qn - 32 + lane];
+                const uint32_t te = pq & 0x7ffu, s = (pq >> 11) & 0x7ffu;
+                const unsigned long long* Rt = Rg + (uint64_t)te * W;
+                const unsigned long long* Rs = Rg + (uint64_t)s * W;
+                if (W == 2) dlr_tail_one<2>(Rt, Rs, Rg, 2, s, tri, k4);
+                else if (W <= 4) dlr_tail_one<4>(Rt, Rs, Rg, W, s, tri, k4);
+                else dlr_tail_one<0>(Rt, Rs, Rg, W, s, tri, k4);
+                qn -= 32;
+                __syncwarp();
+            }
+        }
+        if ((uint32_t)lane < qn) {
+            const uint32_t pq = q_pk[wq][lane];
+            const uint32_t te = pq & 0x7ffu, s = (pq >> 11) & 0x7ffu;
+            const unsigned long long* Rt = Rg + (uint64_t)te * W;
+            const unsigned long long* Rs = Rg + (uint64_t)s * W;
+            if (W == 2) dlr_tail_one<2>(Rt, Rs, Rg, 2, s, tri, k4);
+            else if (W <= 4) dlr_tail_one<4>(Rt, Rs, Rg, W, s, tri, k4);
+            else dlr_tail_one<0>(Rt, Rs, Rg, W, s, tri, k4);
+        }
+        __syncthreads();                                    // srow is free for the next group
+    }
+    tri = warp_sum(tri) * 6ull;
+    k4 = warp_sum(k4) * 24ull;
+    if (lane == 0) {
+        if (tri) atomicAdd(ctrl + kLrLevel, tri);
+        add_u128(ctrl + kCountLo, k4);
     }
 }
 
