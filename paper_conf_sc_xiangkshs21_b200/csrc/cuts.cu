@@ -1012,6 +1012,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
                                 : (wide.n ? k_dlr_tail<false, 3> : k_dlr_tail<false, 0>)));
             kt<<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
                                             (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            CK(cudaGetLastError());
             if (wide.n) {   // the W >= 2 groups: a CTA per group, rows staged by TMA
                 static int occ = 0;
                 if (!occ) {
@@ -1022,6 +1023,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
                 CK(cudaMemsetAsync(ctx->ctrl + kDlrWork, 0, sizeof(unsigned long long), ctx->stream));
                 k_dlr_tail_cta<<<(unsigned)(ctx->num_sms * occ), 256, kDlrSmemBytes, ctx->stream>>>(
                     a, cposb, ea, eb, out, ctx->ctrl, wide, xa, xb);
+                CK(cudaGetLastError());
                 ctx->st.launches++;
             }
             CK(cudaGetLastError());
@@ -1562,6 +1564,8 @@ cuts_status run_query(cuts_ctx* ctx, cuts_mode mode, bool enumerate, uint32_t* r
         ctx->st.count_lo = ctx->h_ctrl[kCountLo];
         ctx->st.count_hi = ctx->h_ctrl[kCountHi];
     }
+    if (ctx->h_ctrl[kErr]) return fail(ctx, CUTS_ECUDA, "internal: %llu deep-rows tail entries out of range",
+                                       (unsigned long long)ctx->h_ctrl[kErr]);
     if (k > 1) ctx->st.level_size[k] = ctx->st.count_lo;
     if (k >= 5) ctx->st.level_size[k - 1] += ctx->h_ctrl[kLrLevel];   // local rows: |L_{k-1}| of the small groups
     ctx->st.alg_bytes_plan = ctx->h_ctrl[kBytesPlan];

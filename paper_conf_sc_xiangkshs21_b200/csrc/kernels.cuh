@@ -1728,7 +1728,7 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
     }
     if (V == 2) {
         if ((uint32_t)lane < qn) dlr_split_item(a.R, q_rb[wq][lane], q_pk[wq][lane], k4);
-    } else if (V) {
+    } else if (V == 1) {
         if (qn) dlr_drain_tri(a.R, (uint32_t)lane < qn ? q_rb[wq][lane] : 0ull, (uint32_t)lane < qn ? q_pk[wq][lane] : 0u,
                               (uint32_t)lane < qn, q_x[V == 1 ? wq : 0], tri, k4);
     } else if ((uint32_t)lane < qn) {
@@ -1775,7 +1775,7 @@ __global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, const uint64_t* __r
     const uint64_t c0 = cpos_b[e0], cbase = a.cpos[a.ea];
     if (threadIdx.x == 0) {
         asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar)));
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
     uint32_t phase = 0;
@@ -1828,8 +1828,10 @@ __global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, const uint64_t* __r
             if (f < F1) {
                 const uint32_t e = out[f].y;
                 const uint32_t te = (uint32_t)(e - g0);
-                const uint32_t s = dlr_select(Rg + (uint64_t)te * W, W, (uint32_t)(f - (cpos_b[e] - c0)));
-                up = te < s;
+                const uint32_t s = te < m ? dlr_select(Rg + (uint64_t)te * W, W, (uint32_t)(f - (cpos_b[e] - c0)))
+                                          : 0xffffffffu;
+                if (s >= m) atomicAdd(ctrl + kErr, 1ull);          // cannot happen: the rows wrote this entry
+                up = te < s && s < m;
                 pk = te | (s << 11) | (W << 22);
             }
             const unsigned bal = __ballot_sync(0xffffffffu, up);

@@ -630,8 +630,9 @@ def test_deep_local_rows_clique_tiers(cuts):
             _set(c, q)
             # the windowed pipeline (no local rows at all) only where its pair count is small
             slow = perm(max(sizes), k - 1) > 2e9
-            for flags in ({}, {"no_cta_tail": True}, {"tail_alt": True}, {"tail_split": True}, {"no_dlr": True}) + \
-                    (() if slow else ({"no_lr": True},)):
+            # the tail variants (ablations) at the large arena only: the small one re-tests chunking
+            variants = ({"no_cta_tail": True}, {"tail_alt": True}, {"tail_split": True}) if arena > (1 << 30) else ()
+            for flags in ({}, {"no_dlr": True}) + variants + (() if slow else ({"no_lr": True},)):
                 c.set_debug(**flags)
                 assert c.count("hybrid") == want, (k, arena, flags)
                 st = c.stats()
