@@ -1367,21 +1367,27 @@ __global__ void __launch_bounds__(256) k_dlr_write(Dlr a, const uint64_t* __rest
     const uint64_t nh = ((uint64_t)gridDim.x * blockDim.x) >> 4;
     for (uint64_t e = e0 + (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 4); e < e1; e += nh) {
         const unsigned long long d = __ldg(a.desc + e);
+        uint64_t o = __ldg(cpos_b + e) - c0;                         // independent of d: issued together
         if (d == ~0ull) continue;                                    // half-warp-uniform
         const uint32_t te = (uint32_t)(d >> 40) & 0x7ffu, m = (uint32_t)(d >> 51) & 0x7ffu;
         const uint64_t g0 = e - te;
         const uint32_t W = (m + 63) / 64;
-        const uint16_t* r = (const uint16_t*)(a.R + (d & ((1ull << 40) - 1)) + (uint64_t)te * W);
-        uint64_t o = __ldg(cpos_b + e) - c0;
-        const uint32_t nsl = (m + 15) / 16;
-        for (uint32_t h = 0; h < nsl; ++h) {
-            const uint32_t x = __ldg(r + h);
-            if (!x) continue;
-            if ((x >> hl) & 1u) {
-                const uint32_t rank = __popc(x & ((1u << hl) - 1u));
-                out[o + rank] = make_uint2(__ldg(&a.lv[g0 + 16u * h + hl].x), (uint32_t)e);
+        const unsigned long long* r = a.R + (d & ((1ull << 40) - 1)) + (uint64_t)te * W;
+        for (uint32_t w = 0; w < W; ++w) {
+            const unsigned long long x = __ldg(r + w);
+            // the four 16-bit slices of the word: member loads issued together, then the stores
+            uint32_t v[4];
+#pragma unroll
+            for (int h = 0; h < 4; ++h) {
+                const bool bit = (x >> (16 * h + hl)) & 1ull;
+                v[h] = bit ? __ldg(&a.lv[g0 + 64u * w + 16u * h + hl].x) : 0u;
             }
-            o += __popc(x);
+#pragma unroll
+            for (int h = 0; h < 4; ++h) {
+                const uint32_t xs = (uint32_t)(x >> (16 * h)) & 0xffffu;
+                if ((xs >> hl) & 1u) out[o + __popc(xs & ((1u << hl) - 1u))] = make_uint2(v[h], (uint32_t)e);
+                o += __popc(xs);
+            }
         }
     }
 }
