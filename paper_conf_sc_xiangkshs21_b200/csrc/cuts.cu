@@ -903,13 +903,14 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
     const uint64_t nscan = std::max<uint64_t>(ng, N) + 1;
     CK(cub::DeviceScan::ExclusiveSum(nullptr, cub_bytes, (uint64_t*)nullptr, (uint64_t*)nullptr, (int64_t)nscan, ctx->stream));
     uint64_t off;
-    TRY(alloc_top(ctx, align_up((ng + 1) * 8) * 2 + align_up((N + 1) * 8) * 3 + align_up(cub_bytes), &off));
+    TRY(alloc_top(ctx, align_up((ng + 1) * 8) * 2 + align_up((N + 1) * 8) * 4 + align_up(cub_bytes), &off));
     char* p = ctx->arena + off;
     uint64_t* rw = (uint64_t*)p; p += align_up((ng + 1) * 8);
     uint64_t* roff = (uint64_t*)p; p += align_up((ng + 1) * 8);
     uint64_t* cnt = (uint64_t*)p; p += align_up((N + 1) * 8);
     uint64_t* cposb = (uint64_t*)p; p += align_up((N + 1) * 8);
     a.desc = (unsigned long long*)p; p += align_up((N + 1) * 8);
+    uint64_t* cposn = (uint64_t*)p; p += align_up((N + 1) * 8);    // split layout: narrow entries' scan
     void* cub_tmp = p;
     int e0 = -1;
     if (timing) { e0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[e0], ctx->stream)); }
@@ -969,6 +970,13 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
     CK(cudaGetLastError());
     CK(cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, cnt, cposb, (int64_t)N + 1, ctx->stream));
     ctx->st.launches += 6;
+    const bool split = wide.n > 0;           // narrow children first, wide after (DlrOut)
+    if (split) {
+        k_dlr_narrow<<<gc, 256, 0, ctx->stream>>>(a, cnt, cnt);   // in place: cnt is not needed after the scan
+        CK(cudaGetLastError());
+        CK(cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, cnt, cposn, (int64_t)N + 1, ctx->stream));
+        ctx->st.launches += 2;
+    }
     if (timing) {
         const int e1 = next_event(ctx);
         CK(cudaEventRecord(ctx->ev_pool[e1], ctx->stream));
@@ -986,13 +994,18 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
         const uint64_t eb = ctx->h_ctrl[kFind], size = ctx->h_ctrl[kFind + 1];
         if (eb <= ea) return fail(ctx, CUTS_ENOMEM, "HYBRID: one level-%d entry's children exceed the arena share", J);
         uint32_t xa = 0, xb = 0;                  // parent slots of the chunk's first and last level-J entry
+        uint64_t nn = 0;                          // split layout: narrow children in the chunk
         if (wide.n && size) {
             CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 2, &a.lv[ea], 8, cudaMemcpyDeviceToHost, ctx->stream));
             CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 3, &a.lv[eb - 1], 8, cudaMemcpyDeviceToHost, ctx->stream));
+            CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 4, cposn + ea, 8, cudaMemcpyDeviceToHost, ctx->stream));
+            CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 5, cposn + eb, 8, cudaMemcpyDeviceToHost, ctx->stream));
             CK(cudaStreamSynchronize(ctx->stream));
             xa = (uint32_t)((ctx->h_ctrl[kCtrlWords + 2] >> 32) - o.w0 - o.ea);
             xb = (uint32_t)((ctx->h_ctrl[kCtrlWords + 3] >> 32) - o.w0 - o.ea);
+            nn = ctx->h_ctrl[kCtrlWords + 5] - ctx->h_ctrl[kCtrlWords + 4];
         }
+        const DlrOut lay{cposb, split ? cposn : nullptr, ea, nn};
         if (size) {
             const uint64_t bot_save = ctx->bot;
             TRY(alloc_bot(ctx, size * sizeof(uint2), &off));
@@ -1000,7 +1013,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
             int t0 = -1;
             if (timing) { t0 = next_event(ctx); CK(cudaEventRecord(ctx->ev_pool[t0], ctx->stream)); }
             const unsigned gw = (unsigned)std::min<uint64_t>((eb - ea + 15) / 16, (uint64_t)ctx->num_sms * 16);   // half-warp per entry
-            k_dlr_write<<<gw, 256, 0, ctx->stream>>>(a, cposb, ea, eb, out);
+            k_dlr_write<<<gw, 256, 0, ctx->stream>>>(a, lay, eb, out);
             CK(cudaGetLastError());
             r.t.lv[J + 1] = out;
             int tm = -1;
@@ -1010,8 +1023,11 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
                           : ((ctx->debug & CUTS_DEBUG_TAIL_ALT) ? k_dlr_tail<false, 1>
                              : ((ctx->debug & CUTS_DEBUG_TAIL_SPLIT) ? k_dlr_tail<false, 2>
                                 : (wide.n ? k_dlr_tail<false, 3> : k_dlr_tail<false, 0>)));
-            kt<<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
-                                            (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            // split: the narrow-group entries [0, nn) with their own scan (k_dlr_tail reads
+            // f - (cposn[e] - cposn[ea])); else the whole chunk with cposb
+            kt<<<split ? (unsigned)std::min<uint64_t>((nn + 255) / 256 + 1, (uint64_t)ctx->num_sms * 16) : gt, 256, 0,
+                 ctx->stream>>>(r.g, r.t, a, split ? cposn : cposb, ea, out, split ? nn : size, ctx->ctrl,
+                                (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
             CK(cudaGetLastError());
             if (wide.n) {   // the W >= 2 groups: a CTA per group, rows staged by TMA
                 static int occ = 0;
@@ -1022,7 +1038,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
                 }
                 CK(cudaMemsetAsync(ctx->ctrl + kDlrWork, 0, sizeof(unsigned long long), ctx->stream));
                 k_dlr_tail_cta<<<(unsigned)(ctx->num_sms * occ), 256, kDlrSmemBytes, ctx->stream>>>(
-                    a, cposb, ea, eb, out, ctx->ctrl, wide, xa, xb);
+                    a, lay, eb, out, ctx->ctrl, wide, xa, xb);
                 CK(cudaGetLastError());
                 ctx->st.launches++;
             }

@@ -1355,21 +1355,47 @@ __global__ void k_dlr_counts(Graph g, Trie t, Dlr a, uint64_t* __restrict__ cnt,
     if (count_bytes) flush_model_bytes(b_plan, b_ext, b_out, b_need, ctrl);
 }
 
+// Where entry e's children sit in the written level-(b+1) chunk (entries [e0, e1)).
+// Plain: cpos[e] - cpos[e0].  Split (with k_dlr_tail_cta): the children of narrow-group
+// entries (W = 1) first, in entry order, then those of wide-group entries — each
+// entry's children still contiguous and ascending — so the warp-queue tail reads only
+// [0, nn) and the CTA tail only [nn, size).  cposn = scan of the narrow entries' child
+// counts; the wide scan is cpos - cposn.
+struct DlrOut {
+    const uint64_t* cpos;
+    const uint64_t* cposn;            // nullptr: plain layout
+    uint64_t e0;
+    uint64_t nn;                      // narrow children in the chunk
+};
+__device__ __forceinline__ uint64_t dlr_child_off(const DlrOut& L, uint64_t e, bool wide) {
+    if (!L.cposn) return L.cpos[e] - L.cpos[L.e0];
+    if (!wide) return L.cposn[e] - L.cposn[L.e0];
+    return L.nn + (L.cpos[e] - L.cposn[e]) - (L.cpos[L.e0] - L.cposn[L.e0]);
+}
+
+// narrow-group entries' child counts (the split layout's first scan)
+__global__ void k_dlr_narrow(Dlr a, const uint64_t* __restrict__ cnt, uint64_t* __restrict__ cntn) {
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e <= a.n; e += (uint64_t)gridDim.x * blockDim.x) {
+        if (e == a.n) { cntn[e] = 0; continue; }
+        const unsigned long long d = a.desc[e];
+        const uint32_t m = d == ~0ull ? 0u : (uint32_t)(d >> 51) & 0x7ffu;
+        cntn[e] = (m > 0 && m <= 64) ? cnt[e] : 0ull;
+    }
+}
+
 // level b+1 written from the rows: entry e's children G[A_e] at its exact offset
 // (ascending, the ordered layout every level of the trie keeps).  A half-warp per entry
 // (two entries in flight per warp): lane i of the half owns member 16h+i of each 16-bit
 // slice h of the row, ranks come from a popcount of the slice below it, so the member
 // reads and the children stores are both coalesced.
-__global__ void __launch_bounds__(256) k_dlr_write(Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0, uint64_t e1,
-                                                   uint2* __restrict__ out) {
-    const uint64_t c0 = __ldg(cpos_b + e0);
+__global__ void __launch_bounds__(256) k_dlr_write(Dlr a, DlrOut L, uint64_t e1, uint2* __restrict__ out) {
     const int lane = threadIdx.x & 31, hl = lane & 15;
     const uint64_t nh = ((uint64_t)gridDim.x * blockDim.x) >> 4;
-    for (uint64_t e = e0 + (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 4); e < e1; e += nh) {
+    for (uint64_t e = L.e0 + (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 4); e < e1; e += nh) {
         const unsigned long long d = __ldg(a.desc + e);
-        uint64_t o = __ldg(cpos_b + e) - c0;                         // independent of d: issued together
         if (d == ~0ull) continue;                                    // half-warp-uniform
         const uint32_t te = (uint32_t)(d >> 40) & 0x7ffu, m = (uint32_t)(d >> 51) & 0x7ffu;
+        uint64_t o = dlr_child_off(L, e, m > 64);
         const uint64_t g0 = e - te;
         const uint32_t W = (m + 63) / 64;
         const unsigned long long* r = a.R + (d & ((1ull << 40) - 1)) + (uint64_t)te * W;
@@ -1768,17 +1794,17 @@ struct DlrWide {                      // parent slots (x = q - ea) of the W >= 2
     uint32_t n;
 };
 
-__global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, const uint64_t* __restrict__ cpos_b, uint64_t e0,
-                                                      uint64_t e1, const uint2* __restrict__ out,
+__global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, DlrOut L, uint64_t e1, const uint2* __restrict__ out,
                                                       unsigned long long* __restrict__ ctrl, DlrWide wide,
                                                       uint32_t xa, uint32_t xb) {
+    const uint64_t e0 = L.e0;
     extern __shared__ __align__(16) unsigned long long srow[];
     __shared__ __align__(8) unsigned long long mbar;
     __shared__ uint32_t q_pk[8][64];
     __shared__ uint64_t s_q;
     unsigned long long tri = 0, k4 = 0;
     const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
-    const uint64_t c0 = cpos_b[e0], cbase = a.cpos[a.ea];
+    const uint64_t cbase = a.cpos[a.ea];
     if (threadIdx.x == 0) {
         asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar)));
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -1806,7 +1832,7 @@ __global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, const uint64_t* __r
         if (W < 2 || m > (uint32_t)kDlrMaxM) { __syncthreads(); continue; }
         const uint64_t t0 = g0 > e0 ? g0 : e0, t1 = (g0 + m < e1) ? g0 + m : e1;
         if (t0 >= t1) { __syncthreads(); continue; }
-        const uint64_t F0 = cpos_b[t0] - c0, F1 = cpos_b[t1] - c0;
+        const uint64_t F0 = dlr_child_off(L, t0, true), F1 = dlr_child_off(L, t1, true);
         const unsigned long long rb = a.roff[q - a.ea];
         const uint32_t bytes = (uint32_t)((((uint64_t)m * W + 1) & ~1ull) * 8);
         const bool staged = bytes <= kDlrSmemBytes;
@@ -1834,7 +1860,7 @@ __global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, const uint64_t* __r
             if (f < F1) {
                 const uint32_t e = out[f].y;
                 const uint32_t te = (uint32_t)(e - g0);
-                const uint32_t s = te < m ? dlr_select(Rg + (uint64_t)te * W, W, (uint32_t)(f - (cpos_b[e] - c0)))
+                const uint32_t s = te < m ? dlr_select(Rg + (uint64_t)te * W, W, (uint32_t)(f - dlr_child_off(L, e, true)))
                                           : 0xffffffffu;
                 if (s >= m) atomicAdd(ctrl + kErr, 1ull);          // cannot happen: the rows wrote this entry
                 up = te < s && s < m;
