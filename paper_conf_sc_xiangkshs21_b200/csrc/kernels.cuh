@@ -23,9 +23,9 @@ namespace cuts {
 constexpr int kMaxK = 8;
 constexpr int kLrMaxM = 512;                // local rows: largest sibling group held in shared memory
 constexpr int kLrWords = kLrMaxM / 32;
-constexpr int kLrBatch = 256;
-constexpr int kDlrMaxM = 1024;
-constexpr uint32_t kDlrSmemBytes = 64u << 10;   // k_dlr_tail_cta: rows staged per group (W >= 2 groups up to this)             // deep local rows: largest sibling group (16 u64 words per row)              // k_lr_group: parent slots claimed per CTA fetch
+constexpr int kLrBatch = 256;              // k_lr_group: parent slots claimed per CTA fetch
+constexpr int kDlrMaxM = 1024;             // deep local rows: largest sibling group (16 u64 words per row)
+constexpr uint32_t kDlrSmemBytes = 32u << 10;   // k_dlr_tail_cta: row blocks staged in shared memory up to this
 constexpr int kTile = 256;   // items per CTA tile == threads per CTA
 
 struct QPlan {                 // query in matching-order positions
