@@ -1794,7 +1794,7 @@ struct DlrWide {                      // parent slots (x = q - ea) of the W >= 2
     uint32_t n;
 };
 
-__global__ void __launch_bounds__(256) k_dlr_tail_cta(Dlr a, DlrOut L, uint64_t e1, const uint2* __restrict__ out,
+__global__ void __launch_bounds__(256, 5) k_dlr_tail_cta(Dlr a, DlrOut L, uint64_t e1, const uint2* __restrict__ out,
                                                       unsigned long long* __restrict__ ctrl, DlrWide wide,
                                                       uint32_t xa, uint32_t xb) {
     const uint64_t e0 = L.e0;
