@@ -950,6 +950,22 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
         CK(cudaStreamSynchronize(ctx->stream));
         wide = DlrWide{wl, (uint32_t)ctx->h_ctrl[kNumSel]};
     }
+    // ... and the 2..64-member groups: k_dlr_tail_narrow's work list
+    DlrWide narrow{nullptr, 0};
+    if (cta_tail && wide.n) {
+        thrust::counting_iterator<uint32_t> it(0);
+        const DlrIsNarrow pred{o.cpos, o.ea};
+        size_t sel_bytes = 0;
+        CK(cub::DeviceSelect::If(nullptr, sel_bytes, it, (uint32_t*)nullptr, ctx->ctrl + kNumSel, (int64_t)ng, pred, ctx->stream));
+        uint64_t noff;
+        TRY(alloc_top(ctx, align_up(std::max<uint64_t>(ng, 1) * 4) + align_up(sel_bytes), &noff));
+        uint32_t* nl = (uint32_t*)(ctx->arena + noff);
+        CK(cub::DeviceSelect::If(ctx->arena + noff + align_up(std::max<uint64_t>(ng, 1) * 4), sel_bytes, it, nl,
+                                 ctx->ctrl + kNumSel, (int64_t)ng, pred, ctx->stream));
+        CK(cudaMemcpyAsync(ctx->h_ctrl + kNumSel, ctx->ctrl + kNumSel, 8, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        narrow = DlrWide{nl, (uint32_t)ctx->h_ctrl[kNumSel]};
+    }
     const double avg = (double)N / (double)std::max<uint64_t>(ng, 1) / 2;     // members tested per entry
     auto go = [&](auto kern, int G) {
         static int occ[4] = {0, 0, 0, 0};
@@ -1022,12 +1038,20 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
             auto kt = cb ? k_dlr_tail<true, 0>
                           : ((ctx->debug & CUTS_DEBUG_TAIL_ALT) ? k_dlr_tail<false, 1>
                              : ((ctx->debug & CUTS_DEBUG_TAIL_SPLIT) ? k_dlr_tail<false, 2>
-                                : (wide.n ? k_dlr_tail<false, 3> : k_dlr_tail<false, 0>)));
+                                : k_dlr_tail<false, 0>));
             // split: the narrow-group entries [0, nn) with their own scan (k_dlr_tail reads
             // f - (cposn[e] - cposn[ea])); else the whole chunk with cposb
-            kt<<<split ? (unsigned)std::min<uint64_t>((nn + 255) / 256 + 1, (uint64_t)ctx->num_sms * 16) : gt, 256, 0,
-                 ctx->stream>>>(r.g, r.t, a, split ? cposn : cposb, ea, out, split ? nn : size, ctx->ctrl,
-                                (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            if (split) {     // the narrow groups: a warp per group, rows in shared memory
+                if (narrow.n && nn) {
+                    CK(cudaMemsetAsync(ctx->ctrl + kDlrWork, 0, sizeof(unsigned long long), ctx->stream));
+                    const unsigned gn = (unsigned)std::min<uint64_t>(((uint64_t)narrow.n + 63) / 64 + 1, (uint64_t)ctx->num_sms * 8);
+                    k_dlr_tail_narrow<<<gn, 256, 0, ctx->stream>>>(a, lay, eb, out, ctx->ctrl, narrow, xa, xb);
+                    ctx->st.launches++;
+                }
+            } else {
+                kt<<<gt, 256, 0, ctx->stream>>>(r.g, r.t, a, cposb, ea, out, size, ctx->ctrl,
+                                                (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
+            }
             CK(cudaGetLastError());
             if (wide.n) {   // the W >= 2 groups: a CTA per group, rows staged by TMA
                 static int occ = 0;

@@ -1223,6 +1223,16 @@ struct DlrIsWide {
     }
 };
 
+// ... and a group with 2..64 members (one row word): k_dlr_tail_narrow's work list
+struct DlrIsNarrow {
+    const uint64_t* cpos;
+    uint64_t ea;
+    __host__ __device__ bool operator()(const uint32_t& x) const {
+        const uint64_t m = cpos[ea + x + 1] - cpos[ea + x];
+        return m >= 2 && m <= 64;
+    }
+};
+
 // per parent slot: row words of its group (0 when it is left to the windowed pipeline)
 __global__ void k_dlr_layout(Dlr a, uint64_t* __restrict__ rw, unsigned long long* __restrict__ ctrl) {
     unsigned long long large = 0;
@@ -1895,6 +1905,76 @@ __global__ void __launch_bounds__(256, 5) k_dlr_tail_cta(Dlr a, DlrOut L, uint64
             else dlr_tail_one<0>(Rt, Rs, Rg, W, s, tri, k4);
         }
         __syncthreads();                                    // srow is free for the next group
+    }
+    tri = warp_sum(tri) * 6ull;
+    k4 = warp_sum(k4) * 24ull;
+    if (lane == 0) {
+        if (tri) atomicAdd(ctrl + kLrLevel, tri);
+        add_u128(ctrl + kCountLo, k4);
+    }
+}
+
+// ---- the tail for narrow groups (2..64 members, one row word): a warp per group ------
+// A warp claims a narrow group, copies its m rows (<= 512 B) into a warp-private slice of
+// shared memory, then walks the group's stored level-(b+1) entries (the narrow part of
+// the split layout) 32 at a time: lane per entry, s by a select on the staged row, and
+// the symmetric 4-clique algebra entirely on shared-memory rows.
+__global__ void __launch_bounds__(256) k_dlr_tail_narrow(Dlr a, DlrOut L, uint64_t e1, const uint2* __restrict__ out,
+                                                         unsigned long long* __restrict__ ctrl, DlrWide narrow,
+                                                         uint32_t xa, uint32_t xb) {
+    __shared__ unsigned long long srow[8][64];
+    unsigned long long tri = 0, k4 = 0;
+    const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
+    const uint64_t e0 = L.e0, cbase = a.cpos[a.ea], n0 = L.cposn[e0];
+    uint32_t lo = 0, hi = narrow.n;
+    {
+        uint32_t l = 0, h = narrow.n;
+        while (l < h) { const uint32_t mid = (l + h) / 2; if (narrow.x[mid] < xa) l = mid + 1; else h = mid; }
+        lo = l;
+        h = narrow.n;
+        while (l < h) { const uint32_t mid = (l + h) / 2; if (narrow.x[mid] <= xb) l = mid + 1; else h = mid; }
+        hi = l;
+    }
+    unsigned long long* rows = srow[wq];
+    for (;;) {
+        unsigned long long i = 0;
+        if (lane == 0) i = lo + atomicAdd(ctrl + kDlrWork, 8ull);          // 8 groups per claim
+        i = __shfl_sync(0xffffffffu, i, 0);
+        if (i >= hi) break;
+        const unsigned long long iend = i + 8 < hi ? i + 8 : hi;
+        for (; i < iend; ++i) {
+            const uint64_t q = a.ea + narrow.x[i];
+            const uint64_t g0 = a.cpos[q] - cbase;
+            const uint32_t m = (uint32_t)(a.cpos[q + 1] - a.cpos[q]);
+            const uint64_t t0 = g0 > e0 ? g0 : e0, t1 = (g0 + m < e1) ? g0 + m : e1;
+            if (t0 >= t1) continue;                                      // warp-uniform
+            const unsigned long long* R = a.R + a.roff[q - a.ea];
+            rows[lane] = (uint32_t)lane < m ? R[lane] : 0ull;
+            rows[lane + 32] = (uint32_t)lane + 32 < m ? R[lane + 32] : 0ull;
+            __syncwarp();
+            const uint64_t F0 = L.cposn[t0] - n0, F1 = L.cposn[t1] - n0;
+            for (uint64_t f = F0 + lane; f - lane < F1; f += 32) {
+                if (f < F1) {
+                    const uint32_t e = out[f].y;
+                    const uint32_t te = (uint32_t)(e - g0);
+                    const unsigned long long At = rows[te & 63];
+                    const uint32_t rank = (uint32_t)(f - (L.cposn[e] - n0));
+                    const uint32_t lo32 = (uint32_t)At, plo = (uint32_t)__popc(lo32);
+                    const uint32_t s = rank < plo ? (uint32_t)__fns(lo32, 0, (int)rank + 1)
+                                                  : 32u + (uint32_t)__fns((uint32_t)(At >> 32), 0, (int)(rank - plo) + 1);
+                    if (te < s && s < 64) {
+                        const unsigned long long x = At & rows[s] & (s == 63u ? 0ull : (~0ull << (s + 1u)));
+                        tri += __popcll(x);
+                        for (unsigned long long y = x; y;) {
+                            const uint32_t l = (uint32_t)(__ffsll((long long)y) - 1);
+                            y &= y - 1;
+                            k4 += __popcll(y & rows[l]);
+                        }
+                    }
+                }
+            }
+            __syncwarp();
+        }
     }
     tri = warp_sum(tri) * 6ull;
     k4 = warp_sum(k4) * 24ull;
