@@ -950,9 +950,23 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
         CK(cudaStreamSynchronize(ctx->stream));
         wide = DlrWide{wl, (uint32_t)ctx->h_ctrl[kNumSel]};
     }
-    // ... and the 2..64-member groups: k_dlr_tail_narrow's work list
-    DlrWide narrow{nullptr, 0};
-    if (cta_tail && wide.n) {
+    // ... and the 2..64- and 65..128-member groups: k_dlr_tail_warp's work lists
+    DlrWide narrow{nullptr, 0}, mid{nullptr, 0};
+    if (cta_tail) {
+        thrust::counting_iterator<uint32_t> it(0);
+        const DlrIsMid pred{o.cpos, o.ea};
+        size_t sel_bytes = 0;
+        CK(cub::DeviceSelect::If(nullptr, sel_bytes, it, (uint32_t*)nullptr, ctx->ctrl + kNumSel, (int64_t)ng, pred, ctx->stream));
+        uint64_t moff;
+        TRY(alloc_top(ctx, align_up(std::max<uint64_t>(ng, 1) * 4) + align_up(sel_bytes), &moff));
+        uint32_t* ml = (uint32_t*)(ctx->arena + moff);
+        CK(cub::DeviceSelect::If(ctx->arena + moff + align_up(std::max<uint64_t>(ng, 1) * 4), sel_bytes, it, ml,
+                                 ctx->ctrl + kNumSel, (int64_t)ng, pred, ctx->stream));
+        CK(cudaMemcpyAsync(ctx->h_ctrl + kNumSel, ctx->ctrl + kNumSel, 8, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        mid = DlrWide{ml, (uint32_t)ctx->h_ctrl[kNumSel]};
+    }
+    if (cta_tail && (wide.n || mid.n)) {
         thrust::counting_iterator<uint32_t> it(0);
         const DlrIsNarrow pred{o.cpos, o.ea};
         size_t sel_bytes = 0;
@@ -986,7 +1000,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
     CK(cudaGetLastError());
     CK(cub::DeviceScan::ExclusiveSum(cub_tmp, cub_bytes, cnt, cposb, (int64_t)N + 1, ctx->stream));
     ctx->st.launches += 6;
-    const bool split = wide.n > 0;           // narrow children first, wide after (DlrOut)
+    const bool split = wide.n > 0 || mid.n > 0;   // narrow children first, wide after (DlrOut)
     if (split) {
         k_dlr_narrow<<<gc, 256, 0, ctx->stream>>>(a, cnt, cnt);   // in place: cnt is not needed after the scan
         CK(cudaGetLastError());
@@ -1011,7 +1025,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
         if (eb <= ea) return fail(ctx, CUTS_ENOMEM, "HYBRID: one level-%d entry's children exceed the arena share", J);
         uint32_t xa = 0, xb = 0;                  // parent slots of the chunk's first and last level-J entry
         uint64_t nn = 0;                          // split layout: narrow children in the chunk
-        if (wide.n && size) {
+        if (split && size) {
             CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 2, &a.lv[ea], 8, cudaMemcpyDeviceToHost, ctx->stream));
             CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 3, &a.lv[eb - 1], 8, cudaMemcpyDeviceToHost, ctx->stream));
             CK(cudaMemcpyAsync(ctx->h_ctrl + kCtrlWords + 4, cposn + ea, 8, cudaMemcpyDeviceToHost, ctx->stream));
@@ -1045,7 +1059,14 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
                 if (narrow.n && nn) {
                     CK(cudaMemsetAsync(ctx->ctrl + kDlrWork, 0, sizeof(unsigned long long), ctx->stream));
                     const unsigned gn = (unsigned)std::min<uint64_t>(((uint64_t)narrow.n + 63) / 64 + 1, (uint64_t)ctx->num_sms * 8);
-                    k_dlr_tail_narrow<<<gn, 256, 0, ctx->stream>>>(a, lay, eb, out, ctx->ctrl, narrow, xa, xb);
+                    k_dlr_tail_warp<1><<<gn, 256, 0, ctx->stream>>>(a, lay, eb, out, ctx->ctrl, narrow, xa, xb);
+                    ctx->st.launches++;
+                }
+                if (mid.n) {
+                    CK(cudaGetLastError());
+                    CK(cudaMemsetAsync(ctx->ctrl + kDlrWork, 0, sizeof(unsigned long long), ctx->stream));
+                    const unsigned gm = (unsigned)std::min<uint64_t>(((uint64_t)mid.n + 15) / 16 + 1, (uint64_t)ctx->num_sms * 8);
+                    k_dlr_tail_warp<2><<<gm, 256, 0, ctx->stream>>>(a, lay, eb, out, ctx->ctrl, mid, xa, xb);
                     ctx->st.launches++;
                 }
             } else {
@@ -1053,7 +1074,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
                                                 (uint32_t)(J + 1), ctx->q.bw[J + 1], ctx->q.bw[J + 2]);
             }
             CK(cudaGetLastError());
-            if (wide.n) {   // the W >= 2 groups: a CTA per group, rows staged by TMA
+            if (wide.n) {   // the W >= 3 groups: a CTA per group, rows staged by TMA
                 static int occ = 0;
                 if (!occ) {
                     cudaFuncSetAttribute(k_dlr_tail_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kDlrSmemBytes);

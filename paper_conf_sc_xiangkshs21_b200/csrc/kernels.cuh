@@ -1219,7 +1219,17 @@ struct DlrIsWide {
     uint64_t ea;
     __host__ __device__ bool operator()(const uint32_t& x) const {
         const uint64_t m = cpos[ea + x + 1] - cpos[ea + x];
-        return m > 64 && m <= (uint64_t)kDlrMaxM;
+        return m > 128 && m <= (uint64_t)kDlrMaxM;
+    }
+};
+
+// ... a group with 65..128 members (two row words): k_dlr_tail_warp<2>'s work list
+struct DlrIsMid {
+    const uint64_t* cpos;
+    uint64_t ea;
+    __host__ __device__ bool operator()(const uint32_t& x) const {
+        const uint64_t m = cpos[ea + x + 1] - cpos[ea + x];
+        return m > 64 && m <= 128;
     }
 };
 
@@ -1839,7 +1849,7 @@ __global__ void __launch_bounds__(256, 5) k_dlr_tail_cta(Dlr a, DlrOut L, uint64
         const uint64_t g0 = a.cpos[q] - cbase;
         const uint32_t m = (uint32_t)(a.cpos[q + 1] - a.cpos[q]);
         const uint32_t W = (m + 63) / 64;
-        if (W < 2 || m > (uint32_t)kDlrMaxM) { __syncthreads(); continue; }
+        if (m <= 128 || m > (uint32_t)kDlrMaxM) { __syncthreads(); continue; }   // W <= 2: k_dlr_tail_warp
         const uint64_t t0 = g0 > e0 ? g0 : e0, t1 = (g0 + m < e1) ? g0 + m : e1;
         if (t0 >= t1) { __syncthreads(); continue; }
         const uint64_t F0 = dlr_child_off(L, t0, true), F1 = dlr_child_off(L, t1, true);
@@ -1914,63 +1924,53 @@ __global__ void __launch_bounds__(256, 5) k_dlr_tail_cta(Dlr a, DlrOut L, uint64
     }
 }
 
-// ---- the tail for narrow groups (2..64 members, one row word): a warp per group ------
-// A warp claims a narrow group, copies its m rows (<= 512 B) into a warp-private slice of
-// shared memory, then walks the group's stored level-(b+1) entries (the narrow part of
-// the split layout) 32 at a time: lane per entry, s by a select on the staged row, and
-// the symmetric 4-clique algebra entirely on shared-memory rows.
-__global__ void __launch_bounds__(256) k_dlr_tail_narrow(Dlr a, DlrOut L, uint64_t e1, const uint2* __restrict__ out,
-                                                         unsigned long long* __restrict__ ctrl, DlrWide narrow,
-                                                         uint32_t xa, uint32_t xb) {
-    __shared__ unsigned long long srow[8][64];
+// ---- the tail for narrow and mid groups: a warp per group --------------------------
+// WM = 1: groups of 2..64 members (one row word; the narrow part of the split layout);
+// WM = 2: 65..128 members (two words; in the wide part).  A warp claims a group, copies
+// its m rows (<= 2 KB) into a warp-private slice of shared memory, then walks the
+// group's stored level-(b+1) entries 32 at a time: lane per entry, s by a select on the
+// staged row, the symmetric 4-clique algebra entirely on shared-memory rows.
+template <int WM>
+__global__ void __launch_bounds__(256) k_dlr_tail_warp(Dlr a, DlrOut L, uint64_t e1, const uint2* __restrict__ out,
+                                                       unsigned long long* __restrict__ ctrl, DlrWide list,
+                                                       uint32_t xa, uint32_t xb) {
+    __shared__ unsigned long long srow[8][64 * WM * WM];
     unsigned long long tri = 0, k4 = 0;
     const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
-    const uint64_t e0 = L.e0, cbase = a.cpos[a.ea], n0 = L.cposn[e0];
-    uint32_t lo = 0, hi = narrow.n;
+    const uint64_t e0 = L.e0, cbase = a.cpos[a.ea];
+    uint32_t lo = 0, hi = list.n;
     {
-        uint32_t l = 0, h = narrow.n;
-        while (l < h) { const uint32_t mid = (l + h) / 2; if (narrow.x[mid] < xa) l = mid + 1; else h = mid; }
+        uint32_t l = 0, h = list.n;
+        while (l < h) { const uint32_t mid = (l + h) / 2; if (list.x[mid] < xa) l = mid + 1; else h = mid; }
         lo = l;
-        h = narrow.n;
-        while (l < h) { const uint32_t mid = (l + h) / 2; if (narrow.x[mid] <= xb) l = mid + 1; else h = mid; }
+        h = list.n;
+        while (l < h) { const uint32_t mid = (l + h) / 2; if (list.x[mid] <= xb) l = mid + 1; else h = mid; }
         hi = l;
     }
     unsigned long long* rows = srow[wq];
     for (;;) {
         unsigned long long i = 0;
-        if (lane == 0) i = lo + atomicAdd(ctrl + kDlrWork, 8ull);          // 8 groups per claim
+        if (lane == 0) i = lo + atomicAdd(ctrl + kDlrWork, (unsigned long long)(WM == 1 ? 8 : 2));
         i = __shfl_sync(0xffffffffu, i, 0);
         if (i >= hi) break;
-        const unsigned long long iend = i + 8 < hi ? i + 8 : hi;
+        const unsigned long long iend = i + (WM == 1 ? 8 : 2) < hi ? i + (WM == 1 ? 8 : 2) : hi;
         for (; i < iend; ++i) {
-            const uint64_t q = a.ea + narrow.x[i];
+            const uint64_t q = a.ea + list.x[i];
             const uint64_t g0 = a.cpos[q] - cbase;
             const uint32_t m = (uint32_t)(a.cpos[q + 1] - a.cpos[q]);
             const uint64_t t0 = g0 > e0 ? g0 : e0, t1 = (g0 + m < e1) ? g0 + m : e1;
             if (t0 >= t1) continue;                                      // warp-uniform
             const unsigned long long* R = a.R + a.roff[q - a.ea];
-            rows[lane] = (uint32_t)lane < m ? R[lane] : 0ull;
-            rows[lane + 32] = (uint32_t)lane + 32 < m ? R[lane + 32] : 0ull;
+            for (uint32_t j = lane; j < 64u * WM * WM; j += 32) rows[j] = j < m * WM ? R[j] : 0ull;
             __syncwarp();
-            const uint64_t F0 = L.cposn[t0] - n0, F1 = L.cposn[t1] - n0;
+            const uint64_t F0 = dlr_child_off(L, t0, WM > 1), F1 = dlr_child_off(L, t1, WM > 1);
             for (uint64_t f = F0 + lane; f - lane < F1; f += 32) {
                 if (f < F1) {
                     const uint32_t e = out[f].y;
                     const uint32_t te = (uint32_t)(e - g0);
-                    const unsigned long long At = rows[te & 63];
-                    const uint32_t rank = (uint32_t)(f - (L.cposn[e] - n0));
-                    const uint32_t lo32 = (uint32_t)At, plo = (uint32_t)__popc(lo32);
-                    const uint32_t s = rank < plo ? (uint32_t)__fns(lo32, 0, (int)rank + 1)
-                                                  : 32u + (uint32_t)__fns((uint32_t)(At >> 32), 0, (int)(rank - plo) + 1);
-                    if (te < s && s < 64) {
-                        const unsigned long long x = At & rows[s] & (s == 63u ? 0ull : (~0ull << (s + 1u)));
-                        tri += __popcll(x);
-                        for (unsigned long long y = x; y;) {
-                            const uint32_t l = (uint32_t)(__ffsll((long long)y) - 1);
-                            y &= y - 1;
-                            k4 += __popcll(y & rows[l]);
-                        }
-                    }
+                    const unsigned long long* Rt = rows + (uint64_t)(te & (64 * WM - 1)) * WM;
+                    const uint32_t s = dlr_select(Rt, WM, (uint32_t)(f - dlr_child_off(L, e, WM > 1)));
+                    if (te < s && s < 64u * WM) dlr_tail_one<WM>(Rt, rows + (uint64_t)s * WM, rows, WM, s, tri, k4);
                 }
             }
             __syncwarp();
