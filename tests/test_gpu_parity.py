@@ -604,7 +604,8 @@ def test_local_rows_group_size_tiers(cuts):
 def test_deep_local_rows_clique_tiers(cuts):
     """Deep local rows (rows of the level-(k-3) sibling groups carry levels k-2, k-1 and
     the count) on clique unions whose level-(k-3) groups span every row width:
-    K6 on K200 ∪ K70 ∪ K9 (groups of 198 / 68 / 7 members: 4-, 2- and 1-word rows),
+    K6 on K200 ∪ K150 ∪ K70 ∪ K9 (groups of 198 / 148 / 68 / 7 members: 4-, 3-, 2- and
+    1-word rows),
     K7 on K70 ∪ K12, K8 on K40 ∪ K11, each plus an ER component (oracle).  In K_n the
     level sizes are n!/(n-j)!.  Default, CUTS_DEBUG_NO_DLR and CUTS_DEBUG_NO_LR agree at
     a large arena and at a 96 MiB one (level k-2 cut into many entry-aligned chunks);
@@ -612,7 +613,7 @@ def test_deep_local_rows_clique_tiers(cuts):
     CUTS_DEBUG_NO_LR only where the windowed pipeline's pair count stays small."""
     from math import perm
     er = er_graph(60, 260, 11)
-    cases = ((6, (200, 70, 9)), (7, (70, 12)), (8, (40, 11)))
+    cases = ((6, (200, 150, 70, 9)), (7, (70, 12)), (8, (40, 11)))
     for k, sizes in cases:
         edges, base = [], 0
         for n in sizes:
