@@ -332,7 +332,7 @@ def run_ours(args):
         # rows, so its roofline is the ALU rate of its unit
         apk, apk_src = _alu_peak()
         ach = tail_ops / (tail_ms / 1e3) / 1e9
-        roof = {"bound": "alu", "kernel": "k_dlr_tail + k_dlr_tail_cta (the deep-rows tail)", "achieved": ach,
+        roof = {"bound": "alu", "kernel": "the deep-rows tail (k_dlr_tail_warp<1|2> + k_dlr_tail_cta)", "achieved": ach,
                 "peak": apk, "unit": "Gword-op/s",
                 "frac": ach / apk, "traffic": ncu.get("dram_bytes_per_launch") if ncu else None,
                 "per_unit": "one 64-bit AND + POPC + add of the symmetric 4-clique bit algebra "
