@@ -933,7 +933,7 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
     CK(cudaMemsetAsync(a.R, 0, words * 8, ctx->stream));
     k_dlr_desc<<<(unsigned)std::min<uint64_t>((N + 255) / 256, (uint64_t)ctx->num_sms * 16), 256, 0, ctx->stream>>>(a);
     CK(cudaGetLastError());
-    // the W >= 2 groups, ascending by parent slot: k_dlr_tail_cta's work list
+    // the 129..1024-member groups, ascending by parent slot: k_dlr_tail_cta's work list
     const bool cta_tail = !cb && !(ctx->debug & (CUTS_DEBUG_TAIL_ALT | CUTS_DEBUG_TAIL_SPLIT | CUTS_DEBUG_NO_CTA_TAIL));
     DlrWide wide{nullptr, 0};
     if (cta_tail) {

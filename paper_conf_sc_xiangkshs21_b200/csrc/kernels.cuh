@@ -1213,7 +1213,8 @@ __global__ void k_dlr_desc(Dlr a) {
     }
 }
 
-// CUB select predicate: parent slot x (window-relative, from ea) owns a group with W >= 2
+// CUB select predicate: parent slot x (window-relative, from ea) owns a group of 129..1024
+// members (k_dlr_tail_cta's work list)
 struct DlrIsWide {
     const uint64_t* cpos;
     uint64_t ea;
@@ -1697,9 +1698,8 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
             const DlrGrp gr = dlr_group(a, e);
             const uint32_t te = (uint32_t)(e - gr.g0);
             const unsigned long long* Rt = a.R + gr.rb + (uint64_t)te * gr.W;
-            const bool mine = !(V == 3 && gr.W >= 2);          // V 3: k_dlr_tail_cta takes W >= 2
-            const uint32_t s = mine ? dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0))) : 0u;
-            up = mine && te < s;
+            const uint32_t s = dlr_select(Rt, gr.W, (uint32_t)(f - (cpos_b[e] - c0)));
+            up = te < s;
             rb = gr.rb;
             pk = te | (s << 11) | (gr.W << 22);
             if (count_bytes) {
@@ -1799,17 +1799,17 @@ __global__ void __launch_bounds__(256) k_dlr_tail(Graph g, Trie t, Dlr a, const 
     }
 }
 
-// ---- the tail for wide-row groups: one CTA per group, the rows staged by TMA ----------
+// ---- the tail for wide groups (129..1024 members): a CTA per group, rows staged by TMA
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
-// Groups with W >= 2 (more than 64 members) hold most of the tail's work and reuse their
-// m x W row block across all their level-(b+1) entries: a CTA takes one such group at a
-// time (dynamic queue over the chunk's parent slots), one elected thread stages the
-// block into shared memory with a single bulk copy (cp.async.bulk, completion on an
-// mbarrier; blocks above kDlrSmemBytes stay in global memory), and the warps run the
-// warp-queue algebra of k_dlr_tail over the group's stored entries with the rows read
-// from shared memory.  Entries of W = 1 groups are left to k_dlr_tail (skip_narrow).
-struct DlrWide {                      // parent slots (x = q - ea) of the W >= 2 groups, ascending (DlrIsWide)
+// Wide groups (129..1024 members, 3..16 row words) hold much of the tail's work and reuse
+// their m x W row block across all their level-(b+1) entries: a CTA takes one such group
+// at a time (dynamic queue over a CUB-selected list of their parent slots), one elected
+// thread stages the block into shared memory with a single bulk copy (cp.async.bulk,
+// completion on an mbarrier; blocks above kDlrSmemBytes stay in global memory), and the
+// warps run the warp-queue algebra of k_dlr_tail over the group's stored entries with
+// the rows read from shared memory.  Smaller groups go to k_dlr_tail_warp.
+struct DlrWide {                      // a work list of parent slots (x = q - ea), ascending (CUB select)
     const uint32_t* __restrict__ x;
     uint32_t n;
 };
