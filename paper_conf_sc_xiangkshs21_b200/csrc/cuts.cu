@@ -990,8 +990,8 @@ cuts_status dlr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large,
         kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, a, ctx->ctrl, batch);
     };
     if (cb) go(k_dlr_rows<16, true>, 16);
-    else if (avg >= 48) go(k_dlr_rows<32, false>, 32);
-    else if (avg >= 12) go(k_dlr_rows<16, false>, 16);
+    else if (avg >= 64) go(k_dlr_rows<32, false>, 32);
+    else if (avg >= 32) go(k_dlr_rows<16, false>, 16);   // C4 (avg 13): 8 lanes beat 16 (1.59 vs 1.64 s)
     else go(k_dlr_rows<8, false>, 8);
     CK(cudaGetLastError());
     const unsigned gc = (unsigned)std::min<uint64_t>((N + 256) / 256, (uint64_t)ctx->num_sms * 16);
