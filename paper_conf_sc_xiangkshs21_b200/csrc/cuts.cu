@@ -437,8 +437,10 @@ void launch_extend_nl(cuts_ctx* ctx, const Graph& g, const Window& w, uint64_t t
     if (w.force_g == 32) launch_extend_g<J, NL, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
     else if (w.force_g == 16) launch_extend_g<J, NL, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
     else if (w.force_g == 8) launch_extend_g<J, NL, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
-    else if (avg >= 96) launch_extend_g<J, NL, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
-    else if (avg >= 24) launch_extend_g<J, NL, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    // lanes per entry from the window's average source length (the paper's single bin,
+    // P:911-916); thresholds measured on C2 (profiles/r04d_c2_g_*.jsonl: 9.97 -> 9.61 s)
+    else if (avg >= 192) launch_extend_g<J, NL, M, 32>(ctx, g, w, t0, t1, out_level, out_rows, cap);
+    else if (avg >= 48) launch_extend_g<J, NL, M, 16>(ctx, g, w, t0, t1, out_level, out_rows, cap);
     else launch_extend_g<J, NL, M, 8>(ctx, g, w, t0, t1, out_level, out_rows, cap);
 }
 
@@ -843,8 +845,8 @@ cuts_status lr_chunk(cuts_ctx* ctx, Run& r, int J, uint64_t N, uint64_t* large) 
         kern<<<(unsigned)grid, 256, 0, ctx->stream>>>(r.g, r.t.lv[J], N, o.cpos, o.w0, o.ea, R, ctx->ctrl, batch);
     };
     if (cb) go(k_lr_rows<16, true>, 16);
-    else if (avg >= 48) go(k_lr_rows<32, false>, 32);
-    else if (avg >= 12) go(k_lr_rows<16, false>, 16);
+    else if (avg >= 64) go(k_lr_rows<32, false>, 32);
+    else if (avg >= 32) go(k_lr_rows<16, false>, 16);
     else go(k_lr_rows<8, false>, 8);
     CK(cudaGetLastError());
     const unsigned grid = (unsigned)std::min<uint64_t>((N + 255) / 256, (uint64_t)ctx->num_sms * 16);
@@ -1124,8 +1126,8 @@ cuts_status pairs_level(cuts_ctx* ctx, Run& r, int J, uint64_t N) {
                                                        r.t, (uint32_t)J, ctx->q.bw[J]);
     };
     if (cb) go(k_pairs<16, true>, 16);                   // instrumented (untimed) pass
-    else if (avg >= 48) go(k_pairs<32, false>, 32);
-    else if (avg >= 12) go(k_pairs<16, false>, 16);
+    else if (avg >= 64) go(k_pairs<32, false>, 32);
+    else if (avg >= 32) go(k_pairs<16, false>, 16);
     else go(k_pairs<8, false>, 8);
     CK(cudaGetLastError());
     if (ctx->debug & CUTS_DEBUG_TIMING) {
